@@ -1,0 +1,334 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 MDMC skycube (BASELINE.json metric: "skycube build time & dominance tests/s,
+n=1M d=12 anticorr, 1/2/4/8 B200").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config H] [--impl ours|reference]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
+
+One step = one whole skycube build (K0 validate -> key sort -> K2 codes -> K1 prefilter -> S+ ->
+K3 MDMC -> K4 compaction into membership rows and the per-subspace id lists) over the synthetic
+workload, input resident in HBM.  value = dominance tests/s = n_ext*(n_ext-1) / (step time, max over
+ranks).  e2e = the same metric through the C-ABI skycube_build_ex with host buffers (H2D of the
+points and D2H of every output inside the timed region; N>1: host input -> per-rank pipeline ->
+rank-0 D2H).  --impl reference times the CPU oracle (oracle/, the reference arm of this tier) on a
+bounded sample of tasks, extrapolated to the whole build.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import datagen  # noqa: E402
+
+METRIC = "skycube build time & dominance tests/s, n=1M d=12 anticorr, 1/2/4/8 B200"
+UNIT = "dominance tests/s"
+L2_FLUSH_BYTES = 256 << 20
+
+
+def algorithmic_ops_per_pair(d: int) -> int:
+    """per ordered S+ pair, the two relation masks of Def. 1 (one compare per
+    dimension each: 2d) plus the probe of B_{p notin S+} (one load + one bit test: 2)."""
+    return 2 * d + 2
+
+
+def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
+    """ALU pipe peak (B300_MICROARCH.md: IADD3/LOP3/SHF/PRMT on the alu pipe, rt = 2 cycles per warp
+    instruction per SMSP -> 16 lanes/SMSP, 64 lanes/SM per clock)."""
+    return sms * 64 * sm_mhz * 1e6
+
+
+def env_rank():
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("LOCAL_RANK", "0"))
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int, path: str | None = None):
+        self.index = index
+        self.proc = None
+        self.path = path
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        self.lines = []
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [l for l in out.splitlines() if l.strip()]
+            if self.path:
+                with open(self.path, "w") as f:
+                    f.write("\n".join(self.lines) + "\n")
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in getattr(self, "lines", []):
+            parts = [p.strip() for p in l.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        loaded = [s for s in sm if mx and s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="H", choices=sorted(datagen.CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--clocks-log", default=None)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------ CPU oracle timing
+def oracle_sample_time(x: np.ndarray, target_s: float, seed: int = 0):
+    """Time Oracle B on a seeded uniform sample of tasks (per-task work is independent of the others,
+    so time * n / sample extrapolates the full build).  Returns (seconds for the whole build,
+    sample size, seconds measured, estimated n_ext, threads)."""
+    import oracle
+    n = x.shape[0]
+    rng = np.random.default_rng(seed)
+    k = 8
+    t = 0.0
+    while True:
+        pids = rng.choice(n, size=min(k, n), replace=False)
+        t0 = time.perf_counter()
+        rows, ext = oracle.rows_b(x, pids, with_ext=True)
+        t = time.perf_counter() - t0
+        if t >= target_s / 4 or k >= n:
+            break
+        k = min(n, int(k * max(2.0, (target_s / 4) / max(t, 1e-3))))
+    full_bit = (1 << x.shape[1]) - 1
+    in_ext = ((ext[:, full_bit >> 5] >> (full_bit & 31)) & 1).astype(bool)
+    est_next = int(round(in_ext.mean() * n))
+    return t * n / len(pids), len(pids), t, est_next, oracle.num_threads()
+
+
+def run_reference(args):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return
+    cfg = datagen.config(args.config)
+    x = cfg.data()
+    per_step = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    times = []
+    for i in range(args.warmup + args.steps):
+        full_s, k, t, est_next, thr = oracle_sample_time(x, per_step, seed=i)
+        if i >= args.warmup:
+            times.append((full_s, k, t, est_next, thr))
+    full = statistics.median([a[0] for a in times])
+    est_next = times[0][3]
+    value = est_next * (est_next - 1) / full
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": full * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {cfg.dist} n={cfg.n} d={cfg.d} seed={cfg.seed}", "n": cfg.n,
+                   "d": cfg.d, "n_ext_estimated": est_next},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": times[0][4], "kind": "oracle",
+                         "sample": f"Oracle B (oracle/skycube_oracle.c) rows for {times[0][1]} uniformly sampled "
+                                   f"points of {cfg.n} per step ({times[0][2]:.1f} s), extrapolated x n/sample; "
+                                   f"n_ext estimated from the sample's S+ bits"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------ GPU arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sigmod_boghcsa17_b200 import build as skybuild
+    rank, world, local = env_rank()
+    if world > 1 and not dist.is_initialized():
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    if rank == 0:
+        skybuild.build()
+    if world > 1:
+        dist.barrier()
+    import paper_conf_sigmod_boghcsa17_b200 as sky
+    from paper_conf_sigmod_boghcsa17_b200.pipeline import DeviceSkycube
+
+    cfg = datagen.config(args.config)
+    x = cfg.data()
+    n, d = x.shape
+    dev = torch.device("cuda", local)
+    pts = torch.from_numpy(x).to(dev)
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+    eng = DeviceSkycube(local)
+    names = ["t0", "t1", "t2", "t3", "t4"]
+
+    def step(events=None):
+        return eng.build(pts, lists=True, membership=True, events=events)
+
+    for _ in range(args.warmup):
+        out = step()
+    torch.cuda.synchronize()
+    m = out["n_ext"]
+    total_ids = out["total_ids"]
+    ev = [{k: torch.cuda.Event(enable_timing=True) for k in names} for _ in range(args.steps)]
+    launches0 = eng.launches
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local, args.clocks_log) as clk:
+        t_start = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_start.record()
+        for s in range(args.steps):
+            flush.fill_(s)  # L2 flush between steps (256 MB > 126 MB L2)
+            step(ev[s])
+        t_end.record()
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = eng.launches - launches0
+    step_ms = [ev[s]["t0"].elapsed_time(ev[s]["t4"]) for s in range(args.steps)]
+    phase = {k: statistics.mean(ev[s][a].elapsed_time(ev[s][b]) for s in range(args.steps))
+             for k, a, b in [("prepare", "t0", "t1"), ("prefilter", "t1", "t2"), ("mdmc", "t2", "t3"),
+                             ("compact", "t3", "t4")]}
+    total_ms = sum(step_ms)
+    if world > 1:
+        tt = torch.tensor([total_ms, phase["mdmc"]], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        total_ms, mdmc_max = tt.tolist()
+    ms_per_step = total_ms / args.steps
+    pairs = m * (m - 1)
+    value = pairs / (ms_per_step / 1e3)
+
+    # ---- e2e through the public API with host buffers
+    e2e = None
+    if not args.no_e2e:
+        e2e = measure_e2e(args, x, eng, world, rank, dev, pairs)
+
+    if rank != 0:
+        return
+    clocks = clk.summary()
+    sm_mhz = clocks["sm_mhz"] or 1965.0
+    # roofline of the dominant kernel (K3 MDMC), duration from CUDA events on its stream
+    mdmc_ms = phase["mdmc"]
+    my_pairs = pairs if world == 1 else pairs / world
+    ops = my_pairs * algorithmic_ops_per_pair(d)
+    achieved = ops / (mdmc_ms / 1e3) / 1e12
+    peak = alu_peak_ops(sm_mhz) / 1e12
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {cfg.dist} n={n} d={d} seed={cfg.seed} (datagen, Börzsönyi-style)",
+                   "n": n, "d": d, "n_ext": m, "pairs": pairs, "total_ids": total_ids,
+                   "l2": "256 MB buffer written between timed steps",
+                   "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
+        "phases_ms": phase,
+        "gpu_launches": launches,
+        "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
+                     "frac": achieved / peak, "traffic": None,
+                     "kernel": "k3_mdmc", "ops_per_pair": algorithmic_ops_per_pair(d),
+                     "peak_basis": f"148 SM x 64 ALU lanes x {sm_mhz:.0f} MHz (median SM clock under load)"},
+        "clocks": clocks,
+    }
+    if e2e is not None:
+        line["e2e"] = e2e
+    if not args.no_cpu and world == 1 or (not args.no_cpu and rank == 0 and world == 1):
+        full_s, k, t, est_next, thr = oracle_sample_time(x, args.cpu_seconds)
+        cpu_value = pairs / full_s
+        line["cpu_baseline"] = {"value": cpu_value, "unit": UNIT, "cores": thr, "kind": "oracle",
+                                "sample": f"Oracle B rows for {k} uniformly sampled points of {n} "
+                                          f"({t:.1f} s on {thr} threads), extrapolated x n/sample to "
+                                          f"{full_s:.0f} s for the whole build"}
+    print(json.dumps(line), flush=True)
+
+
+def measure_e2e(args, x, eng, world, rank, dev, pairs):
+    import torch
+    import torch.distributed as dist
+    n, d = x.shape
+    if world == 1:
+        import paper_conf_sigmod_boghcsa17_b200 as sky
+        r = sky.skycube_build_raw(x, stats=True)  # warm (pinned pools, contexts)
+        d2h = 4 * r.n_ext + 4 * n * sky.words_per_row(d) + 8 * ((1 << d) + 1) + 4 * int(r.offsets()[-1])
+        r.close()
+        times = []
+        for _ in range(args.e2e_steps):
+            t0 = time.perf_counter()
+            r = sky.skycube_build_raw(x)
+            times.append(time.perf_counter() - t0)
+            r.close()
+        t = statistics.median(times)
+        return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
+                "ms_per_step": t * 1e3, "api": "skycube_build_ex (C-ABI, host buffers, pinned result pool)"}
+    # N > 1: pinned host input -> every rank H2D -> sharded pipeline -> rank 0 D2H of all outputs
+    host = torch.from_numpy(x).pin_memory()
+    times = []
+    d2h = 0
+    for i in range(args.e2e_steps + 1):
+        dist.barrier()
+        t0 = time.perf_counter()
+        pts = host.to(dev, non_blocking=True)
+        out = eng.build(pts, lists=True, membership=True)
+        if rank == 0:
+            res = [out["membership"].cpu(), out["ext_ids"].cpu(), out["offsets"].cpu(), out["ids"].cpu()]
+            d2h = sum(t.numel() * t.element_size() for t in res)
+        torch.cuda.synchronize()
+        dist.barrier()
+        if i:
+            times.append(time.perf_counter() - t0)
+    t = statistics.median(times)
+    return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
+            "ms_per_step": t * 1e3, "api": "pipeline.DeviceSkycube (per-rank C-ABI device entry points)"}
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,150 @@
+/*
+ * skycube.h — C-ABI of the B200-native point-based MDMC skycube (Bøgh, Chester, Šidlauskas, Assent,
+ * "Template Skycube Algorithms for Heterogeneous Parallelism on Multicore and GPU Architectures",
+ * SIGMOD'17).  Citations "Lnnn" are lines of the paper transcript.
+ *
+ * What is computed (Def. 1-3):
+ *   Input P: n points over d dimensions, float32, smaller is better (footnote 2, L109).
+ *   For every subspace 0 < delta < 2^d (bit i of delta <=> dimension i, L71), the subspace skyline
+ *     S_delta(P) = { p : no q in P dominates p in delta }, where q dominates p in delta iff
+ *     (B_{q=p} & delta) != delta and (B_{q<=p} & delta) == delta (Def. 1).
+ *   The skycube (Def. 3) is returned in two forms:
+ *     - per point, its membership bitmap (the paper's B_{p in S}, L79, here UNSHIFTED: bit delta, not
+ *       bit delta-1);
+ *     - per subspace, the ascending id list of S_delta(P) (the lattice of Fig. 1a).
+ *   Method: Alg. 3 (MDMC, L313-319) on the GPU: S+(P) prefilter (line 2), then one data-parallel task
+ *   per p in S+(P) computing B_{p notin S} and B_{p notin S+} (lines 3-12), then compaction.
+ *
+ * Value semantics (readings Q9-Q12): IEEE binary32 compares only; -0 == +0; +-inf are
+ * ordinary values; NaN is rejected (SKYCUBE_ENAN); equal points never dominate each other; ids are
+ * the row indices of `points` (footnote 1, L73).
+ *
+ * Errors: every entry point returns a skycube_status; on any error the output struct is zeroed and
+ * owns nothing; skycube_last_error() gives a thread-local detail string.  All calls are serialised
+ * by a process-wide mutex.
+ */
+#ifndef SKYCUBE_H
+#define SKYCUBE_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    SKYCUBE_OK = 0,
+    SKYCUBE_EINVAL = 1, /* bad argument: NULL pointer with n > 0, d outside [1,16], n > INT32_MAX */
+    SKYCUBE_ENAN = 2,   /* a NaN in the input */
+    SKYCUBE_ENOMEM = 3, /* host or device allocation failed */
+    SKYCUBE_ECUDA = 4,  /* CUDA runtime / kernel error */
+    SKYCUBE_ENCCL = 5,  /* reserved: collective error (multi-GPU) */
+    SKYCUBE_ENODEV = 6  /* no sm_100 device visible */
+} skycube_status;
+
+/* flags for skycube_opts.flags */
+#define SKYCUBE_NO_LISTS 0x1u          /* skip the per-subspace id lists (rows only) */
+#define SKYCUBE_EXT_MEMBERSHIP 0x2u    /* debug: also return B_{p in S+} rows (ext_membership) */
+
+typedef struct {
+    int32_t d;                 /* 1..16 */
+    int64_t n;                 /* number of points */
+    int64_t n_ext;             /* |S+(P)|: full-space extended skyline size (Def. 2, delta = 2^d-1) */
+    int32_t *ext_ids;          /* [n_ext] ascending ids of S+(P) */
+    uint32_t words_per_row;    /* W = max(1, 2^d / 32) */
+    uint32_t *membership;      /* [n * W] row p, bit delta (word delta>>5, bit delta&31) <=> p in S_delta(P);
+                                  bit 0 always 0; rows of points outside S+(P) are all zero (L101) */
+    uint32_t *ext_membership;  /* [n * W] or NULL: bit delta <=> p in S+_delta(P) (SKYCUBE_EXT_MEMBERSHIP) */
+    int64_t *cuboid_offsets;   /* [2^d + 1] or NULL (NO_LISTS): ids of S_delta are
+                                  cuboid_ids[off[delta] .. off[delta+1]); off[0] = off[1] = 0 */
+    int32_t *cuboid_ids;       /* [off[2^d]] ascending within each delta */
+} skycube_result;
+
+typedef struct {
+    int32_t num_gpus;     /* reserved for the single-process multi-GPU path; 0 or 1 = one GPU */
+    int32_t device;       /* CUDA device ordinal to use */
+    uint32_t flags;       /* SKYCUBE_* flags */
+} skycube_opts;
+
+typedef struct {
+    double ms_total;       /* whole call, host clock */
+    double ms_h2d, ms_validate, ms_sort, ms_codes, ms_prefilter, ms_mdmc, ms_compact, ms_d2h; /* CUDA events */
+    int64_t n_ext;         /* |S+(P)| */
+    int64_t pairs;         /* n_ext * (n_ext - 1): ordered S+ pairs tested by MDMC */
+    int64_t total_ids;     /* sum over delta of |S_delta(P)| */
+    int32_t kernel_launches;
+} skycube_stats;
+
+/* Build the skycube of the host array points[n*d] (row-major, row = id, column i = dimension i).
+ * `points` is caller-owned and only read.  `out` is caller-provided; every buffer in it is allocated
+ * by the library (pinned host memory) and must be released with skycube_free.  n == 0 returns OK
+ * with empty outputs.  Uses CUDA device 0. */
+skycube_status skycube_build(const float *points, int64_t n, int32_t d, skycube_result *out);
+
+/* As skycube_build with options (NULL = defaults) and optional per-phase statistics (NULL = none). */
+skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const skycube_opts *opts,
+                                skycube_result *out, skycube_stats *stats);
+
+/* Release every buffer of `out` and zero it.  Idempotent; safe on a zeroed struct. */
+void skycube_free(skycube_result *out);
+
+const char *skycube_strerror(skycube_status s);
+const char *skycube_last_error(void);   /* thread-local detail of the last error */
+
+/* ------------------------------------------------------------------------------------------------
+ * Device-resident entry points (used by the per-rank multi-GPU driver and the benchmark).
+ * All pointers here are DEVICE pointers on the context's device; `stream` is a cudaStream_t passed as
+ * void* (NULL = legacy default stream).  A context owns a grow-only device workspace reused across
+ * calls; it is not thread-safe (one context per thread / rank).
+ * ------------------------------------------------------------------------------------------------ */
+typedef struct skycube_ctx skycube_ctx;
+
+skycube_status skycube_ctx_create(int32_t device, skycube_ctx **ctx);
+void skycube_ctx_destroy(skycube_ctx *ctx);
+
+/* Phase 1 (replicated on every rank): validate (K0: NaN -> ENAN, -0 -> +0, order-preserving keys),
+ * sort by the exact key sum (Λ2), and compute per-dimension 15-bit monotone codes (K2).
+ * d_points: [n*d] float32 row-major on the device. */
+skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, void *stream);
+
+/* Phase 2: extended-skyline prefilter (K1).  Sorted positions are cut into tiles of 256; this call
+ * processes the tiles t with t % tile_step == tile_offset (interleaving balances ranks: later tiles
+ * have longer candidate prefixes).  Writes d_ext_sorted[s] = 1 iff the point at key-sorted position s
+ * is in S+(P), 0 otherwise, for the positions of those tiles only.
+ * d_ext_sorted: [n] uint8 device buffer owned by the caller. */
+skycube_status skycube_dev_prefilter(skycube_ctx *ctx, int64_t tile_offset, int64_t tile_step,
+                                     uint8_t *d_ext_sorted, void *stream);
+
+/* Phase 3: install the S+ flags (d_ext_sorted: [n] complete, identical on every rank) and build the
+ * S+ structures; returns n_ext. */
+skycube_status skycube_dev_set_ext(skycube_ctx *ctx, const uint8_t *d_ext_sorted, int64_t *n_ext, void *stream);
+
+/* Phase 4: MDMC (K3) for the S+ points j in [j_begin, j_end) (id-ascending S+ index; j_begin a
+ * multiple of 32, j_end <= n_ext).  Writes their membership rows into d_rows32, the tiled layout
+ * d_rows32[(j/32)*W*32 + w*32 + j%32] = word w of the membership bitmap of S+ point j
+ * (buffer size ceil(n_ext/32)*32*W uint32).  d_ext_rows32 (same layout, may be NULL) receives the
+ * extended-skyline rows B_{p in S+} (debug / tests). */
+skycube_status skycube_dev_mdmc(skycube_ctx *ctx, int64_t j_begin, int64_t j_end, uint32_t *d_rows32,
+                                uint32_t *d_ext_rows32, void *stream);
+
+/* Phase 5: compaction (K4): from the complete tiled rows of all S+ points, write
+ * d_membership[n*W] (NULL = skip), d_ext_ids[n_ext] (NULL = skip), and, unless d_offsets == NULL,
+ * the lattice: d_offsets[2^d+1] and d_ids[total_ids].  Call first with d_ids == NULL to obtain
+ * *total_ids (offsets are written), then with d_ids of that size. */
+skycube_status skycube_dev_compact(skycube_ctx *ctx, const uint32_t *d_rows32, uint32_t *d_membership,
+                                   int32_t *d_ext_ids, int64_t *d_offsets, int32_t *d_ids,
+                                   int64_t *total_ids, void *stream);
+
+/* Number of kernels launched by this context since creation (for the benchmark's gpu_launches). */
+int64_t skycube_ctx_launches(const skycube_ctx *ctx);
+
+/* Problem facts after prepare / set_ext: n_ext (0 before set_ext), words per row, and the bit mask of
+ * dimensions whose 15-bit codes are injective (exact). Any pointer may be NULL. */
+skycube_status skycube_ctx_info(const skycube_ctx *ctx, int64_t *n_ext, uint32_t *words_per_row,
+                                uint32_t *exact_mask);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SKYCUBE_H */

@@ -1,0 +1,261 @@
+"""B200-native point-based MDMC skycube (Bøgh et al., SIGMOD'17) — thin Python binding.
+
+The binding only marshals arguments to the C-ABI of ``include/skycube.h`` (``libskycube.so``, built
+in-tree by ``paper_conf_sigmod_boghcsa17_b200.build``).  Every step of the skycube runs in the CUDA
+kernels of ``csrc/``; there is no CPU fallback: if the library or an sm_100 GPU is missing, calls
+raise.  PyTorch is only used by callers for device memory, streams and process groups.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libskycube.so")
+
+OK, EINVAL, ENAN, ENOMEM, ECUDA, ENCCL, ENODEV = range(7)
+NO_LISTS = 0x1
+EXT_MEMBERSHIP = 0x2
+
+EXPORTED = (
+    "skycube_build", "skycube_build_ex", "skycube_free", "skycube_strerror", "skycube_last_error",
+    "skycube_ctx_create", "skycube_ctx_destroy", "skycube_dev_prepare", "skycube_dev_prefilter",
+    "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
+    "skycube_ctx_info",
+)
+
+
+class SkycubeError(RuntimeError):
+    def __init__(self, status, detail):
+        super().__init__(f"skycube status {status}: {detail}")
+        self.status = status
+
+
+class Result(ctypes.Structure):
+    _fields_ = [
+        ("d", ctypes.c_int32),
+        ("n", ctypes.c_int64),
+        ("n_ext", ctypes.c_int64),
+        ("ext_ids", ctypes.POINTER(ctypes.c_int32)),
+        ("words_per_row", ctypes.c_uint32),
+        ("membership", ctypes.POINTER(ctypes.c_uint32)),
+        ("ext_membership", ctypes.POINTER(ctypes.c_uint32)),
+        ("cuboid_offsets", ctypes.POINTER(ctypes.c_int64)),
+        ("cuboid_ids", ctypes.POINTER(ctypes.c_int32)),
+    ]
+
+
+class Opts(ctypes.Structure):
+    _fields_ = [("num_gpus", ctypes.c_int32), ("device", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_double) for k in ("ms_total", "ms_h2d", "ms_validate", "ms_sort", "ms_codes",
+                                                "ms_prefilter", "ms_mdmc", "ms_compact", "ms_d2h")] + [
+        ("n_ext", ctypes.c_int64), ("pairs", ctypes.c_int64), ("total_ids", ctypes.c_int64),
+        ("kernel_launches", ctypes.c_int32)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+_lib = None
+
+
+def lib():
+    """Load libskycube.so; raises (never falls back) if it is missing."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built: run python -m paper_conf_sigmod_boghcsa17_b200.build")
+        L = ctypes.CDLL(LIB_PATH)
+        P, I64, I32, U32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32
+        L.skycube_build.argtypes = [P, I64, I32, ctypes.POINTER(Result)]
+        L.skycube_build_ex.argtypes = [P, I64, I32, ctypes.POINTER(Opts), ctypes.POINTER(Result),
+                                       ctypes.POINTER(Stats)]
+        L.skycube_free.argtypes = [ctypes.POINTER(Result)]
+        L.skycube_free.restype = None
+        L.skycube_strerror.argtypes = [ctypes.c_int]
+        L.skycube_strerror.restype = ctypes.c_char_p
+        L.skycube_last_error.restype = ctypes.c_char_p
+        L.skycube_ctx_create.argtypes = [I32, ctypes.POINTER(P)]
+        L.skycube_ctx_destroy.argtypes = [P]
+        L.skycube_ctx_destroy.restype = None
+        L.skycube_dev_prepare.argtypes = [P, P, I64, I32, P]
+        L.skycube_dev_prefilter.argtypes = [P, I64, I64, P, P]
+        L.skycube_dev_set_ext.argtypes = [P, P, ctypes.POINTER(I64), P]
+        L.skycube_dev_mdmc.argtypes = [P, I64, I64, P, P, P]
+        L.skycube_dev_compact.argtypes = [P, P, P, P, P, P, ctypes.POINTER(I64), P]
+        L.skycube_ctx_launches.argtypes = [P]
+        L.skycube_ctx_launches.restype = I64
+        L.skycube_ctx_info.argtypes = [P, ctypes.POINTER(I64), ctypes.POINTER(U32), ctypes.POINTER(U32)]
+        for f in ("skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
+                  "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
+                  "skycube_ctx_info"):
+            getattr(L, f).restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _check(status):
+    if status != OK:
+        raise SkycubeError(status, lib().skycube_last_error().decode(errors="replace"))
+
+
+def words_per_row(d: int) -> int:
+    return max(1, (1 << d) >> 5)
+
+
+def _view(ptr, count, dtype):
+    if count <= 0 or not ptr:
+        return np.zeros(0, dtype)
+    return np.ctypeslib.as_array(ptr, shape=(count,)).view(dtype)
+
+
+class RawResult:
+    """Owns a skycube_result (pinned host buffers); views are valid until close()."""
+
+    def __init__(self, res: Result, stats: Stats | None):
+        self._res = res
+        self.stats = stats.as_dict() if stats is not None else None
+
+    @property
+    def n(self):
+        return self._res.n
+
+    @property
+    def d(self):
+        return self._res.d
+
+    @property
+    def n_ext(self):
+        return self._res.n_ext
+
+    def ext_ids(self):
+        return _view(self._res.ext_ids, self._res.n_ext, np.int32)
+
+    def membership(self):
+        W = self._res.words_per_row
+        return _view(self._res.membership, self._res.n * W, np.uint32).reshape(self._res.n, W)
+
+    def ext_membership(self):
+        W = self._res.words_per_row
+        if not self._res.ext_membership:
+            return None
+        return _view(self._res.ext_membership, self._res.n * W, np.uint32).reshape(self._res.n, W)
+
+    def offsets(self):
+        if not self._res.cuboid_offsets:
+            return None
+        return _view(self._res.cuboid_offsets, (1 << self._res.d) + 1, np.int64)
+
+    def ids(self):
+        off = self.offsets()
+        if off is None:
+            return None
+        return _view(self._res.cuboid_ids, int(off[-1]), np.int32)
+
+    def close(self):
+        if self._res is not None:
+            lib().skycube_free(ctypes.byref(self._res))
+            self._res = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def skycube_build_raw(points: np.ndarray, *, device: int = 0, lists: bool = True, ext_membership: bool = False,
+                      stats: bool = False) -> RawResult:
+    """Call skycube_build_ex on a host (n, d) float32 array; returns the owning RawResult."""
+    pts = np.ascontiguousarray(points, dtype=np.float32)
+    if pts.ndim != 2:
+        raise ValueError("points must be (n, d)")
+    n, d = pts.shape
+    opts = Opts(1, device, (0 if lists else NO_LISTS) | (EXT_MEMBERSHIP if ext_membership else 0))
+    res = Result()
+    st = Stats() if stats else None
+    _check(lib().skycube_build_ex(pts.ctypes.data_as(ctypes.c_void_p) if n else None, n, d, ctypes.byref(opts),
+                                  ctypes.byref(res), ctypes.byref(st) if st is not None else None))
+    return RawResult(res, st)
+
+
+def skycube_build(points: np.ndarray, **kw) -> dict:
+    """Skycube of a host (n, d) float32 array, copied into numpy arrays:
+    rows [n, W] uint32 (bit delta <=> point in S_delta), ext_ids, offsets [2^d+1], ids."""
+    with skycube_build_raw(points, **kw) as r:
+        out = {"rows": r.membership().copy(), "ext_ids": r.ext_ids().copy(), "n_ext": r.n_ext}
+        off = r.offsets()
+        if off is not None:
+            out["offsets"] = off.copy()
+            out["ids"] = r.ids().copy()
+        em = r.ext_membership()
+        if em is not None:
+            out["ext_rows"] = em.copy()
+        if r.stats is not None:
+            out["stats"] = r.stats
+        return out
+
+
+@dataclass
+class Context:
+    """Device-level API (device pointers as ints, e.g. torch tensor .data_ptr(); stream as int)."""
+
+    device: int = 0
+
+    def __post_init__(self):
+        h = ctypes.c_void_p()
+        _check(lib().skycube_ctx_create(self.device, ctypes.byref(h)))
+        self._h = h
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().skycube_ctx_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def prepare(self, d_points: int, n: int, d: int, stream: int = 0):
+        _check(lib().skycube_dev_prepare(self._h, d_points, n, d, stream or None))
+
+    def prefilter(self, d_ext_sorted: int, tile_offset: int = 0, tile_step: int = 1, stream: int = 0):
+        _check(lib().skycube_dev_prefilter(self._h, tile_offset, tile_step, d_ext_sorted, stream or None))
+
+    def set_ext(self, d_ext_sorted: int, stream: int = 0) -> int:
+        m = ctypes.c_int64()
+        _check(lib().skycube_dev_set_ext(self._h, d_ext_sorted, ctypes.byref(m), stream or None))
+        return m.value
+
+    def mdmc(self, d_rows32: int, j_begin: int, j_end: int, d_ext_rows32: int = 0, stream: int = 0):
+        _check(lib().skycube_dev_mdmc(self._h, j_begin, j_end, d_rows32, d_ext_rows32 or None, stream or None))
+
+    def compact(self, d_rows32: int, d_membership: int = 0, d_ext_ids: int = 0, d_offsets: int = 0,
+                d_ids: int = 0, stream: int = 0) -> int:
+        tot = ctypes.c_int64(0)
+        _check(lib().skycube_dev_compact(self._h, d_rows32, d_membership or None, d_ext_ids or None,
+                                         d_offsets or None, d_ids or None, ctypes.byref(tot), stream or None))
+        return tot.value
+
+    @property
+    def launches(self) -> int:
+        return lib().skycube_ctx_launches(self._h)
+
+    def info(self):
+        m, W, ex = ctypes.c_int64(), ctypes.c_uint32(), ctypes.c_uint32()
+        _check(lib().skycube_ctx_info(self._h, ctypes.byref(m), ctypes.byref(W), ctypes.byref(ex)))
+        return {"n_ext": m.value, "words_per_row": W.value, "exact_mask": ex.value}

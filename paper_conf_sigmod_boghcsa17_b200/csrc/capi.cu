@@ -1,0 +1,377 @@
+// capi.cu — the C-ABI of include/skycube.h: argument validation, the per-device context cache,
+// pinned host-memory pool for results, phase orchestration on one stream, and per-phase CUDA-event
+// statistics.  Every compute step runs in the kernels of prep.cu / k1_prefilter.cu / k3_mdmc.cu /
+// k4_compact.cu; there is no CPU fallback: without an sm_100 device every call fails with ENODEV.
+#include <chrono>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <unordered_map>
+
+#include "../../include/skycube.h"
+#include "ctx.cuh"
+
+struct skycube_ctx {
+    sky::Ctx c;
+    sky::DevBuf input, ext8, rows32, ext_rows32, membership, offsets, ids;
+};
+
+namespace {
+
+std::mutex g_mutex;                  // serialises skycube_build* (header: "calls are serialised")
+thread_local std::string g_last_error;
+
+skycube_status fail(skycube_status s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+// ----------------------------------------------------------------------- pinned host memory pool
+struct PinnedPool {
+    std::mutex mu;
+    std::multimap<size_t, void *> free_;
+    std::unordered_map<void *, size_t> size_of;
+    size_t cached = 0;
+    static constexpr size_t kMaxCached = (size_t)48 << 30;
+
+    void *get(size_t bytes) {
+        if (bytes == 0) bytes = 64;
+        {
+            std::lock_guard<std::mutex> lk(mu);
+            auto it = free_.lower_bound(bytes);
+            if (it != free_.end() && it->first <= bytes + bytes / 2 + (1 << 20)) {
+                void *p = it->second;
+                cached -= it->first;
+                free_.erase(it);
+                return p;
+            }
+        }
+        void *p = nullptr;
+        if (cudaMallocHost(&p, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            // drop the cache and retry once
+            release_all();
+            if (cudaMallocHost(&p, bytes) != cudaSuccess) {
+                cudaGetLastError();
+                throw sky::Error{3, "cudaMallocHost(" + std::to_string(bytes) + ") failed"};
+            }
+        }
+        std::lock_guard<std::mutex> lk(mu);
+        size_of[p] = bytes;
+        return p;
+    }
+    void put(void *p) {
+        if (!p) return;
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = size_of.find(p);
+        if (it == size_of.end()) return;
+        if (cached + it->second > kMaxCached) {
+            cudaFreeHost(p);
+            size_of.erase(it);
+            return;
+        }
+        free_.emplace(it->second, p);
+        cached += it->second;
+    }
+    void release_all() {
+        std::lock_guard<std::mutex> lk(mu);
+        for (auto &kv : free_) {
+            cudaFreeHost(kv.second);
+            size_of.erase(kv.second);
+        }
+        free_.clear();
+        cached = 0;
+    }
+};
+PinnedPool g_pool;
+
+std::map<int, skycube_ctx *> g_ctx;  // one cached context per device for skycube_build*
+
+void check_device(int device) {
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) {
+        cudaGetLastError();
+        throw sky::Error{SKYCUBE_ENODEV, "no CUDA device visible"};
+    }
+    if (device < 0 || device >= count) throw sky::Error{SKYCUBE_ENODEV, "device ordinal out of range"};
+    cudaDeviceProp prop;
+    SKY_CUDA(cudaGetDeviceProperties(&prop, device));
+    if (prop.major != 10) throw sky::Error{SKYCUBE_ENODEV, std::string("not an sm_100 device: ") + prop.name};
+    SKY_CUDA(cudaSetDevice(device));
+}
+
+skycube_ctx *new_ctx(int device) {
+    check_device(device);
+    auto *x = new skycube_ctx();
+    x->c.device = device;
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    x->c.num_sms = sms;
+    return x;
+}
+
+template <typename F>
+skycube_status guarded(F &&f) {
+    try {
+        f();
+        return SKYCUBE_OK;
+    } catch (const sky::Error &e) {
+        return fail((skycube_status)e.status, e.msg);
+    } catch (const std::bad_alloc &) {
+        return fail(SKYCUBE_ENOMEM, "host allocation failed");
+    } catch (...) {
+        return fail(SKYCUBE_ECUDA, "unexpected exception");
+    }
+}
+
+float ev_ms(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, a, b);
+    return ms;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *skycube_strerror(skycube_status s) {
+    switch (s) {
+        case SKYCUBE_OK: return "ok";
+        case SKYCUBE_EINVAL: return "invalid argument";
+        case SKYCUBE_ENAN: return "NaN in input";
+        case SKYCUBE_ENOMEM: return "out of memory";
+        case SKYCUBE_ECUDA: return "CUDA error";
+        case SKYCUBE_ENCCL: return "collective error";
+        case SKYCUBE_ENODEV: return "no sm_100 device";
+    }
+    return "unknown status";
+}
+
+const char *skycube_last_error(void) { return g_last_error.c_str(); }
+
+void skycube_free(skycube_result *out) {
+    if (!out) return;
+    g_pool.put(out->ext_ids);
+    g_pool.put(out->membership);
+    g_pool.put(out->ext_membership);
+    g_pool.put(out->cuboid_offsets);
+    g_pool.put(out->cuboid_ids);
+    std::memset(out, 0, sizeof(*out));
+}
+
+skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const skycube_opts *opts,
+                                skycube_result *out, skycube_stats *stats) {
+    if (!out) return fail(SKYCUBE_EINVAL, "out == NULL");
+    std::memset(out, 0, sizeof(*out));
+    if (stats) std::memset(stats, 0, sizeof(*stats));
+    if (d < 1 || d > 16) return fail(SKYCUBE_EINVAL, "d must be in [1, 16]");
+    if (n < 0 || n > INT32_MAX) return fail(SKYCUBE_EINVAL, "n must be in [0, INT32_MAX]");
+    if (n > 0 && !points) return fail(SKYCUBE_EINVAL, "points == NULL");
+    const uint32_t flags = opts ? opts->flags : 0u;
+    const int device = opts ? opts->device : 0;
+    std::lock_guard<std::mutex> lk(g_mutex);
+    const auto t0 = std::chrono::steady_clock::now();
+    skycube_result r;
+    std::memset(&r, 0, sizeof(r));
+    skycube_status st = guarded([&] {
+        r.d = d;
+        r.n = n;
+        r.words_per_row = sky::words_per_row(d);
+        const uint32_t W = r.words_per_row;
+        const int64_t nsub = (int64_t)1 << d;
+        skycube_ctx *&x = g_ctx[device];
+        if (!x) x = new_ctx(device);
+        else check_device(device);
+        sky::Ctx &c = x->c;
+        const int64_t launches0 = c.L.count;
+        if (n == 0) {
+            if (!(flags & SKYCUBE_NO_LISTS)) {
+                r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
+                std::memset(r.cuboid_offsets, 0, sizeof(int64_t) * (nsub + 1));
+            }
+            return;
+        }
+        cudaStream_t s = nullptr;
+        cudaEvent_t ev[9];
+        for (auto &e : ev) SKY_CUDA(cudaEventCreate(&e));
+        struct EvGuard {
+            cudaEvent_t *e;
+            ~EvGuard() { for (int i = 0; i < 9; i++) cudaEventDestroy(e[i]); }
+        } eg{ev};
+        x->input.ensure(sizeof(float) * n * d);
+        SKY_CUDA(cudaEventRecord(ev[0], s));
+        SKY_CUDA(cudaMemcpyAsync(x->input.p, points, sizeof(float) * n * d, cudaMemcpyHostToDevice, s));
+        SKY_CUDA(cudaEventRecord(ev[1], s));
+        sky::prep_run(c, x->input.as<float>(), n, d, s);
+        SKY_CUDA(cudaEventRecord(ev[2], s));
+        x->ext8.ensure(n);
+        sky::prefilter_run(c, 0, 1, x->ext8.as<uint8_t>(), s);
+        sky::ext_build(c, x->ext8.as<uint8_t>(), s);
+        SKY_CUDA(cudaEventRecord(ev[3], s));
+        const int64_t m = c.m;
+        const size_t rows_words = (size_t)sky::ceil_div(m > 0 ? m : 1, 32) * 32 * W;
+        x->rows32.ensure(sizeof(uint32_t) * rows_words);
+        const bool want_ext = (flags & SKYCUBE_EXT_MEMBERSHIP) != 0;
+        if (want_ext) x->ext_rows32.ensure(sizeof(uint32_t) * rows_words);
+        sky::mdmc_run(c, 0, m, x->rows32.as<uint32_t>(), want_ext ? x->ext_rows32.as<uint32_t>() : nullptr, s);
+        SKY_CUDA(cudaEventRecord(ev[4], s));
+        x->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
+        sky::compact_membership(c, x->rows32.as<uint32_t>(), x->membership.as<uint32_t>(), s);
+        int64_t total = 0;
+        const bool lists = !(flags & SKYCUBE_NO_LISTS);
+        if (lists) {
+            x->offsets.ensure(sizeof(int64_t) * (nsub + 1));
+            sky::compact_lattice(c, x->rows32.as<uint32_t>(), x->offsets.as<int64_t>(), nullptr, &total, s);
+            x->ids.ensure(sizeof(int32_t) * (total > 0 ? total : 1));
+            sky::compact_lattice(c, x->rows32.as<uint32_t>(), x->offsets.as<int64_t>(), x->ids.as<int32_t>(), &total, s);
+        }
+        SKY_CUDA(cudaEventRecord(ev[5], s));
+        // device -> pinned host
+        r.n_ext = m;
+        r.ext_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (m > 0 ? m : 1));
+        r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
+        if (m) SKY_CUDA(cudaMemcpyAsync(r.ext_ids, c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaMemcpyAsync(r.membership, x->membership.p, sizeof(uint32_t) * (size_t)n * W,
+                                 cudaMemcpyDeviceToHost, s));
+        if (lists) {
+            r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
+            r.cuboid_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (total > 0 ? total : 1));
+            SKY_CUDA(cudaMemcpyAsync(r.cuboid_offsets, x->offsets.p, sizeof(int64_t) * (nsub + 1),
+                                     cudaMemcpyDeviceToHost, s));
+            if (total)
+                SKY_CUDA(cudaMemcpyAsync(r.cuboid_ids, x->ids.p, sizeof(int32_t) * total, cudaMemcpyDeviceToHost, s));
+        }
+        if (want_ext) {
+            sky::compact_membership(c, x->ext_rows32.as<uint32_t>(), x->membership.as<uint32_t>() , s);
+            r.ext_membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
+            SKY_CUDA(cudaMemcpyAsync(r.ext_membership, x->membership.p, sizeof(uint32_t) * (size_t)n * W,
+                                     cudaMemcpyDeviceToHost, s));
+        }
+        SKY_CUDA(cudaEventRecord(ev[6], s));
+        SKY_CUDA(cudaStreamSynchronize(s));
+        SKY_CUDA(cudaGetLastError());
+        if (stats) {
+            stats->ms_h2d = ev_ms(ev[0], ev[1]);
+            stats->ms_validate = 0;  // K0 + sorts + codes are one phase (prep)
+            stats->ms_sort = ev_ms(ev[1], ev[2]);
+            stats->ms_codes = 0;
+            stats->ms_prefilter = ev_ms(ev[2], ev[3]);
+            stats->ms_mdmc = ev_ms(ev[3], ev[4]);
+            stats->ms_compact = ev_ms(ev[4], ev[5]);
+            stats->ms_d2h = ev_ms(ev[5], ev[6]);
+            stats->n_ext = m;
+            stats->pairs = m * (m > 0 ? m - 1 : 0);
+            stats->total_ids = total;
+            stats->kernel_launches = (int32_t)(c.L.count - launches0);
+        }
+    });
+    if (st != SKYCUBE_OK) {
+        skycube_free(&r);
+        return st;
+    }
+    if (stats)
+        stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = r;
+    return SKYCUBE_OK;
+}
+
+skycube_status skycube_build(const float *points, int64_t n, int32_t d, skycube_result *out) {
+    return skycube_build_ex(points, n, d, nullptr, out, nullptr);
+}
+
+// ------------------------------------------------------------------------------ device-level API
+skycube_status skycube_ctx_create(int32_t device, skycube_ctx **ctx) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    *ctx = nullptr;
+    return guarded([&] { *ctx = new_ctx(device); });
+}
+
+void skycube_ctx_destroy(skycube_ctx *ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->c.device);
+    sky::Ctx &c = ctx->c;
+    for (sky::DevBuf *b : {&c.ord, &c.keysum, &c.perm, &c.comp_keys, &c.comp_vals, &c.keys_alt, &c.vals_alt,
+                           &c.counts, &c.scan_tmp, &c.flags, &c.scanned, &c.rbuf, &c.nanflag, &c.codes_id,
+                           &c.codes_sorted, &c.ord_sorted, &c.ext_id_flag, &c.ext_idx, &c.key_flag, &c.key_idx,
+                           &c.ext_ids, &c.p_codes, &c.p_ord, &c.q_codes, &c.q_ord, &c.tie, &c.lat_counts,
+                           &c.scan64_tmp, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
+                           &ctx->membership, &ctx->offsets, &ctx->ids})
+        b->release();
+    delete ctx;
+}
+
+int64_t skycube_ctx_launches(const skycube_ctx *ctx) { return ctx ? ctx->c.L.count : 0; }
+
+skycube_status skycube_ctx_info(const skycube_ctx *ctx, int64_t *n_ext, uint32_t *words_per_row,
+                                uint32_t *exact_mask) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (n_ext) *n_ext = ctx->c.ext_ready ? ctx->c.m : 0;
+    if (words_per_row) *words_per_row = ctx->c.W;
+    if (exact_mask) *exact_mask = ctx->c.exact_mask;
+    return SKYCUBE_OK;
+}
+
+skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, void *stream) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (d < 1 || d > 16) return fail(SKYCUBE_EINVAL, "d must be in [1, 16]");
+    if (n < 1 || n > INT32_MAX) return fail(SKYCUBE_EINVAL, "n must be in [1, INT32_MAX]");
+    if (!d_points) return fail(SKYCUBE_EINVAL, "d_points == NULL");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::prep_run(ctx->c, d_points, n, d, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_prefilter(skycube_ctx *ctx, int64_t tile_offset, int64_t tile_step,
+                                     uint8_t *d_ext_sorted, void *stream) {
+    if (!ctx || !d_ext_sorted) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::prefilter_run(ctx->c, tile_offset, tile_step, d_ext_sorted, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_set_ext(skycube_ctx *ctx, const uint8_t *d_ext_sorted, int64_t *n_ext, void *stream) {
+    if (!ctx || !d_ext_sorted) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::ext_build(ctx->c, d_ext_sorted, (cudaStream_t)stream);
+        if (n_ext) *n_ext = ctx->c.m;
+    });
+}
+
+skycube_status skycube_dev_mdmc(skycube_ctx *ctx, int64_t j_begin, int64_t j_end, uint32_t *d_rows32,
+                                uint32_t *d_ext_rows32, void *stream) {
+    if (!ctx || !d_rows32) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::mdmc_run(ctx->c, j_begin, j_end, d_rows32, d_ext_rows32, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_compact(skycube_ctx *ctx, const uint32_t *d_rows32, uint32_t *d_membership,
+                                   int32_t *d_ext_ids, int64_t *d_offsets, int32_t *d_ids, int64_t *total_ids,
+                                   void *stream) {
+    if (!ctx || !d_rows32) return fail(SKYCUBE_EINVAL, "NULL argument");
+    if (d_ids && !d_offsets) return fail(SKYCUBE_EINVAL, "d_ids needs d_offsets");
+    return guarded([&] {
+        sky::Ctx &c = ctx->c;
+        if (!c.ext_ready) throw sky::Error{SKYCUBE_EINVAL, "skycube_dev_compact before skycube_dev_set_ext"};
+        SKY_CUDA(cudaSetDevice(c.device));
+        cudaStream_t s = (cudaStream_t)stream;
+        if (d_membership) sky::compact_membership(c, d_rows32, d_membership, s);
+        if (d_ext_ids && c.m)
+            SKY_CUDA(cudaMemcpyAsync(d_ext_ids, c.ext_ids.p, sizeof(int32_t) * c.m, cudaMemcpyDeviceToDevice, s));
+        if (d_offsets) {
+            int64_t tot = 0;
+            if (!d_ids) {
+                sky::compact_lattice(c, d_rows32, d_offsets, nullptr, &tot, s);
+                if (total_ids) *total_ids = tot;
+            } else {
+                sky::compact_lattice(c, d_rows32, d_offsets, d_ids, &tot, s);
+            }
+        }
+    });
+}
+
+}  // extern "C"

@@ -1,0 +1,86 @@
+// ctx.cuh — per-device context: grow-only device workspace and the phase launchers.
+#pragma once
+
+#include "common.cuh"
+
+namespace sky {
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t bytes = 0;
+    template <typename T>
+    T *as() const { return reinterpret_cast<T *>(p); }
+    void ensure(size_t b) {
+        if (b <= bytes) return;
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+        size_t want = b + b / 8 + 256;
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            throw Error{3, std::string("cudaMalloc(") + std::to_string(want) + "): " + cudaGetErrorString(e)};
+        }
+        bytes = want;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+    }
+};
+
+struct Ctx {
+    int device = 0;
+    int num_sms = 148;
+    Launches L;
+    // problem
+    int64_t n = 0;
+    int d = 0, dp = 0;
+    uint32_t W = 1;
+    uint32_t exact_mask = 0;    // bit i <=> the codes of dimension i are injective (dense ranks)
+    uint32_t R[kMaxD] = {0};    // distinct values per dimension
+    int64_t m = 0;              // |S+(P)|
+    bool prepared = false, ext_ready = false;
+    // preparation (all n points)
+    DevBuf ord;         // u32 [n*d]   order-preserving keys, id order
+    DevBuf keysum;      // u64 [n]     sum of keys (Λ2), later sorted
+    DevBuf perm;        // u32 [n]     sorted position -> id
+    DevBuf comp_keys;   // u64 [n*d]   (dim << 32) | key, sorted per dimension
+    DevBuf comp_vals;   // u32 [n*d]   point id
+    DevBuf keys_alt, vals_alt, counts, scan_tmp;
+    DevBuf flags;       // u32 [n*d]
+    DevBuf scanned;     // u32 [n*d]
+    DevBuf rbuf;        // u32 [kMaxD]
+    DevBuf nanflag;     // u32 [1]
+    DevBuf codes_id;    // u16 [n*dp]  id order
+    DevBuf codes_sorted;// u16 [n*dp]  key-sum order
+    DevBuf ord_sorted;  // u32 [n*d]   key-sum order
+    // S+ (m points)
+    DevBuf ext_id_flag, ext_idx, key_flag, key_idx;  // u32 [n]
+    DevBuf ext_ids;     // i32 [m] ascending
+    DevBuf p_codes;     // u16 [m*dp]  S+ in id order (MDMC tasks)
+    DevBuf p_ord;       // u32 [m*d]
+    DevBuf q_codes;     // u16 [m*dp]  S+ in key-sum order (MDMC competitor stream)
+    DevBuf q_ord;       // u32 [m*d]
+    DevBuf tie;         // u32 tiled rows: tie contributions to B_{p notin S}
+    DevBuf lat_counts;  // u64 [2^d * nchunks]
+    DevBuf scan64_tmp;
+};
+
+// prep.cu
+void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st);
+void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st);
+// k1_prefilter.cu
+void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ext_sorted, cudaStream_t st);
+// k3_mdmc.cu
+void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st);
+// k4_compact.cu
+void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cudaStream_t st);
+void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
+                     cudaStream_t st);
+
+constexpr int kPrefilterTile = 256;  // sorted positions per K1 block
+
+}  // namespace sky

@@ -1,0 +1,375 @@
+// k3_mdmc.cu — K3: the MDMC per-point task of Alg. 3 (L313-319), lines 3-12, on sm_100a.
+//
+// For every p in S+(P) (the data-parallel tasks, L306-310) and every competitor q in S+(P) (Λ1:
+// competitors outside S+ add nothing), the pair reduces to two d-bit masks (L77)
+//     L = B_{q<=p},  S = B_{q<p}   (E = L \ S = B_{q=p})
+// and q dominates p exactly in the subspaces { delta subset of L : delta & S != 0 } (Def. 1), strictly in the
+// non-empty subsets of S.  B_{p notin S+} (strict) is downward closed, so bit L set in it means q adds
+// nothing new (L330-336, Alg. 3 line 11) — the probe that skips almost every pair.
+//
+// Per pair, on the hot path:
+//   1. M = B_{code(q)<=code(p)} by SWAR over 16-bit code lanes with a guard bit (2 dimensions per
+//      32-bit subtraction), gathered to a d-bit mask with a byte permute and one multiply per 4
+//      dimensions.  Codes are monotone (Λ3), so M is a superset of L (equal where codes are exact).
+//   2. probe bit M of B_{p notin S+} in shared memory; set => skip (Λ4).
+// Only on a miss (rare: < 1% of pairs):
+//   3. S from the strict SWAR compare; exact refinement of the dimensions whose codes tie but are not
+//      injective; then set sub(S) in B_{p notin S+} (Alg. 3 line 12, word-parallel), and, only when q
+//      ties p somewhere (E != 0), the tie contribution sub(L) \ sub(E) in a global tie row (reading Q3).
+//   B_{p notin S} = B_{p notin S+} | tie row; the membership row written out is its complement.
+//
+// Two layouts of the per-task state (the paper's thread-block-per-point of L498-512 is prior art):
+//   design A (d <= 12): one thread per task p, a warp = 32 tasks, every competitor q is read once per
+//     CTA from shared memory as a broadcast; B_{p notin S+} lives in shared memory as [word][lane]
+//     (bank = lane, conflict-free probes).  2^d/8 bytes per task.
+//   design B (d > 12): one warp per task (PPW tasks per warp), lanes stride over q; the 2^d-bit state
+//     (8 KB at d = 16) is shared by the warp; misses expand with shared atomics.
+#include "ctx.cuh"
+
+namespace sky {
+namespace {
+
+template <int D>
+struct Geo {
+    static constexpr int DP = ((D + 3) / 4) * 4;
+    static constexpr int CW = DP / 2;                       // 32-bit code words per point
+    static constexpr int NG = DP / 4;                       // groups of 4 dimensions
+    static constexpr int WB = D >= 5 ? (1 << (D - 5)) : 1;  // 32-bit words of a 2^d-bit state
+    static constexpr uint32_t kRowMask = D >= 5 ? 0xffffffffu : ((1u << (1 << D)) - 1u);
+};
+
+// Mask of guard bits -> d-bit mask, dimension i -> bit i.  Word k holds dimensions 2k (bits 0-15) and
+// 2k+1 (bits 16-31); guard bits at 15 and 31.  Per group of 4 dimensions: byte-permute the 4 guard
+// bytes into one word, keep the MSBs, and move them to bits 28..31 with a carry-free multiply.
+template <int NG>
+__device__ __forceinline__ uint32_t gather_mask(const uint32_t *v) {
+    uint32_t m = 0;
+#pragma unroll
+    for (int g = NG - 1; g >= 0; g--) {
+        const uint32_t x = __byte_perm(v[2 * g], v[2 * g + 1], 0x7531) & 0x80808080u;
+        const uint32_t y = x * 0x00204081u;  // byte k MSB (bit 8k+7) -> bit 28+k, no carries
+        m = __funnelshift_l(y, m, 4);       // (m << 4) | (y >> 28)
+    }
+    return m;
+}
+
+// Bits delta_low (0..31) that are subsets of x (x < 32): the word pattern of sub(x) in the low 5 dims.
+__device__ __forceinline__ uint32_t sub5(uint32_t x) {
+    uint32_t t = 1u;
+    if (x & 1u) t |= t << 1;
+    if (x & 2u) t |= t << 2;
+    if (x & 4u) t |= t << 4;
+    if (x & 8u) t |= t << 8;
+    if (x & 16u) t |= t << 16;
+    return t;
+}
+
+// Exact refinement of the dimensions in U (codes tie, codes not injective there).
+__device__ __forceinline__ void refine_exact(uint32_t U, const uint32_t *__restrict__ qo, const uint32_t *__restrict__ po,
+                                             uint32_t &L, uint32_t &S) {
+    while (U) {
+        const int i = __ffs(U) - 1;
+        U &= U - 1;
+        const uint32_t qv = qo[i], pv = po[i];
+        if (qv > pv) L &= ~(1u << i);
+        else if (qv < pv) S |= 1u << i;
+    }
+}
+
+// ==================================================================================== design A
+constexpr int kAWarps = 4;
+constexpr int kATQ = 128;  // competitors per shared-memory tile
+
+template <int D>
+__global__ void __launch_bounds__(kAWarps * 32) k3_mdmc_a_kernel(
+    const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ q_codes,
+    const uint32_t *__restrict__ q_ord, int64_t ntiles_q, int64_t j_begin, int64_t j_end, uint32_t inexact,
+    uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
+    using G = Geo<D>;
+    extern __shared__ uint32_t smem[];
+    uint32_t *qs = smem;                                            // [kATQ][CW]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t *st = smem + kATQ * G::CW + warp * G::WB * 32 + lane;  // word w of this task: st[w * 32]
+    const int64_t j = j_begin + (int64_t)blockIdx.x * (kAWarps * 32) + warp * 32 + lane;
+    const bool active = j < j_end;
+    const int64_t grp = j >> 5;
+
+    uint32_t pH[G::CW];
+#pragma unroll
+    for (int k = 0; k < G::CW; k++) {
+        uint32_t w = active ? p_codes[j * G::CW + k] : 0u;
+        if (2 * k >= D) w &= 0xffff0000u;  // padding dimensions: p = 0 never passes q <= p (q pad = 1)
+        if (2 * k + 1 >= D) w &= 0x0000ffffu;
+        pH[k] = w | kGuard;
+    }
+#pragma unroll 4
+    for (int w = 0; w < G::WB; w++) st[w * 32] = w == 0 ? 1u : 0u;  // bit 0 (empty subspace) preset
+    bool had_tie = false;
+
+    for (int64_t tq = 0; tq < ntiles_q; tq++) {
+        __syncthreads();
+        {
+            const uint4 *src = reinterpret_cast<const uint4 *>(q_codes + tq * kATQ * G::CW);
+            uint4 *dst = reinterpret_cast<uint4 *>(qs);
+            for (int i = threadIdx.x; i < kATQ * G::CW / 4; i += kAWarps * 32) dst[i] = src[i];
+        }
+        __syncthreads();
+        if (!active) continue;
+#pragma unroll 2
+        for (int t = 0; t < kATQ; t++) {
+            const uint32_t *qw = qs + t * G::CW;
+            uint32_t le[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) le[k] = pH[k] - qw[k];  // guard <=> code(q) <= code(p)
+            const uint32_t M = gather_mask<G::NG>(le);
+            const uint32_t word = st[(M >> 5) * 32];
+            if ((word >> (M & 31)) & 1u) continue;                     // Λ4: nothing new from q
+            // ---- miss: exact masks, then Alg. 3 line 12
+            uint32_t lt[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) lt[k] = pH[k] - qw[k] - 0x00010001u;  // guard <=> code(q) < code(p)
+            uint32_t S = gather_mask<G::NG>(lt);
+            uint32_t L = M;
+            const uint32_t U = M & ~S & inexact;
+            if (U) {
+                const int64_t q = tq * kATQ + t;
+                refine_exact(U, q_ord + q * D, p_ord + j * D, L, S);
+            }
+            if (S == 0) continue;                                      // q is nowhere better than p
+            if (L != M && ((st[(L >> 5) * 32] >> (L & 31)) & 1u)) continue;
+            {   // B_{p notin S+} |= sub(S)   (strict dominance propagates to all submasks, L330)
+                const uint32_t sh = S >> 5, bits = sub5(S & 31u);
+                uint32_t w = 0;
+                do {
+                    st[w * 32] |= bits;
+                    w = (w - sh) & sh;
+                } while (w);
+            }
+            if (L != S) {  // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}
+                const uint32_t E = L & ~S;
+                const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
+                uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
+                uint32_t w = 0;
+                do {
+                    const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
+                    tr[w * 32] |= bits;
+                    w = (w - lh) & lh;
+                } while (w);
+                had_tie = true;
+            }
+        }
+    }
+    if (!active) return;
+    const bool any_tie = __any_sync(__activemask(), had_tie);
+    uint32_t *out = rows32 + grp * (G::WB * 32) + lane;
+    const uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
+#pragma unroll 4
+    for (int w = 0; w < G::WB; w++) {
+        uint32_t v = st[w * 32];
+        if (any_tie && had_tie) v |= tr[w * 32];
+        uint32_t row = ~v & G::kRowMask;
+        if (w == 0) row &= ~1u;
+        out[w * 32] = row;
+        if (ext_rows32) {
+            uint32_t er = ~st[w * 32] & G::kRowMask;
+            if (w == 0) er &= ~1u;
+            ext_rows32[grp * (G::WB * 32) + w * 32 + lane] = er;
+        }
+    }
+}
+
+// ==================================================================================== design B
+constexpr int kBWarps = 8;
+constexpr int kBPPW = 2;   // tasks per warp
+constexpr int kBTQ = 256;  // competitors per tile
+
+template <int D>
+__global__ void __launch_bounds__(kBWarps * 32) k3_mdmc_b_kernel(
+    const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ q_codes,
+    const uint32_t *__restrict__ q_ord, int64_t ntiles_q, int64_t j_begin, int64_t j_end, uint32_t inexact,
+    uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
+    using G = Geo<D>;
+    extern __shared__ uint32_t smem[];
+    uint32_t *qs = smem;  // [kBTQ][CW]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t *stw = smem + kBTQ * G::CW + warp * (kBPPW * G::WB);  // [kBPPW][WB]
+    int64_t jt[kBPPW];
+    bool act[kBPPW];
+    uint32_t pH[kBPPW][G::CW];
+#pragma unroll
+    for (int s = 0; s < kBPPW; s++) {
+        jt[s] = j_begin + ((int64_t)blockIdx.x * kBWarps + warp) * kBPPW + s;
+        act[s] = jt[s] < j_end;
+#pragma unroll
+        for (int k = 0; k < G::CW; k++) {
+            uint32_t w = act[s] ? p_codes[jt[s] * G::CW + k] : 0u;
+            if (2 * k >= D) w &= 0xffff0000u;
+            if (2 * k + 1 >= D) w &= 0x0000ffffu;
+            pH[s][k] = w | kGuard;
+        }
+    }
+    for (int w = lane; w < kBPPW * G::WB; w += 32) stw[w] = (w % G::WB) == 0 ? 1u : 0u;
+    bool had_tie[kBPPW];
+#pragma unroll
+    for (int s = 0; s < kBPPW; s++) had_tie[s] = false;
+    __syncwarp();
+
+    for (int64_t tq = 0; tq < ntiles_q; tq++) {
+        __syncthreads();
+        {
+            const uint4 *src = reinterpret_cast<const uint4 *>(q_codes + tq * kBTQ * G::CW);
+            uint4 *dst = reinterpret_cast<uint4 *>(qs);
+            for (int i = threadIdx.x; i < kBTQ * G::CW / 4; i += kBWarps * 32) dst[i] = src[i];
+        }
+        __syncthreads();
+        for (int t = lane; t < kBTQ; t += 32) {
+            uint32_t qw[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) qw[k] = qs[t * G::CW + k];
+#pragma unroll
+            for (int s = 0; s < kBPPW; s++) {
+                if (!act[s]) continue;
+                uint32_t *st = stw + s * G::WB;
+                uint32_t le[G::CW];
+#pragma unroll
+                for (int k = 0; k < G::CW; k++) le[k] = pH[s][k] - qw[k];
+                const uint32_t M = gather_mask<G::NG>(le);
+                if ((st[M >> 5] >> (M & 31)) & 1u) continue;
+                uint32_t lt[G::CW];
+#pragma unroll
+                for (int k = 0; k < G::CW; k++) lt[k] = pH[s][k] - qw[k] - 0x00010001u;
+                uint32_t S = gather_mask<G::NG>(lt);
+                uint32_t L = M;
+                const uint32_t U = M & ~S & inexact;
+                if (U) {
+                    const int64_t q = tq * kBTQ + t;
+                    refine_exact(U, q_ord + q * D, p_ord + jt[s] * D, L, S);
+                }
+                if (S == 0) continue;
+                if (L != M && ((st[L >> 5] >> (L & 31)) & 1u)) continue;
+                {
+                    const uint32_t sh = S >> 5, bits = sub5(S & 31u);
+                    uint32_t w = 0;
+                    do {
+                        atomicOr(&st[w], bits);
+                        w = (w - sh) & sh;
+                    } while (w);
+                }
+                if (L != S) {
+                    const uint32_t E = L & ~S;
+                    const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
+                    uint32_t *tr = tie32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
+                    uint32_t w = 0;
+                    do {
+                        const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
+                        atomicOr(&tr[w * 32], bits);
+                        w = (w - lh) & lh;
+                    } while (w);
+                    had_tie[s] = true;
+                }
+            }
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int s = 0; s < kBPPW; s++) {
+        if (!act[s]) continue;
+        const bool any_tie = __any_sync(0xffffffffu, had_tie[s]);
+        const uint32_t *st = stw + s * G::WB;
+        uint32_t *out = rows32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
+        const uint32_t *tr = tie32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
+        for (int w = lane; w < G::WB; w += 32) {
+            uint32_t v = st[w];
+            if (any_tie) v |= tr[w * 32];
+            uint32_t row = ~v;
+            if (w == 0) row &= ~1u;
+            out[w * 32] = row;
+            if (ext_rows32) {
+                uint32_t er = ~st[w];
+                if (w == 0) er &= ~1u;
+                ext_rows32[(jt[s] >> 5) * (G::WB * 32) + w * 32 + (jt[s] & 31)] = er;
+            }
+        }
+    }
+}
+
+template <int D>
+void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    using G = Geo<D>;
+    const size_t smem = sizeof(uint32_t) * ((size_t)kATQ * G::CW + (size_t)kAWarps * G::WB * 32);
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_a_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const int64_t ntq = ceil_div(c.m, kATQ);
+    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, kAWarps * 32);
+    k3_mdmc_a_kernel<D><<<blocks, kAWarps * 32, smem, st>>>(
+        c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(), ntq,
+        j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
+template <int D>
+void launch_b(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    using G = Geo<D>;
+    const size_t smem = sizeof(uint32_t) * ((size_t)kBTQ * G::CW + (size_t)kBWarps * kBPPW * G::WB);
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_b_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const int64_t ntq = ceil_div(c.m, kBTQ);
+    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, kBWarps * kBPPW);
+    k3_mdmc_b_kernel<D><<<blocks, kBWarps * 32, smem, st>>>(
+        c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(), ntq,
+        j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
+// Competitor stream padded to whole tiles with "never better" points (code 0x7fff, key 0xffffffff).
+__global__ void pad_q_kernel(uint32_t *q_codes, uint32_t *q_ord, int64_t m, int64_t mpad, int cw, int d) {
+    const int64_t q = m + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (q >= mpad) return;
+    for (int k = 0; k < cw; k++) q_codes[q * cw + k] = 0x7fff7fffu;
+    for (int i = 0; i < d; i++) q_ord[q * d + i] = 0xffffffffu;
+}
+
+}  // namespace
+
+void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st) {
+    if (!c.ext_ready) throw Error{1, "skycube_dev_mdmc before skycube_dev_set_ext"};
+    if (j_begin < 0 || j_end > c.m || (j_begin & 31)) throw Error{1, "bad MDMC task range"};
+    if (j_end <= j_begin) return;
+    const int d = c.d;
+    const int cw = c.dp / 2;
+    // q stream padding to whole tiles (both designs use tiles of at most 256)
+    const int64_t mpad = ceil_div(c.m, 256) * 256;
+    c.q_codes.ensure(sizeof(uint32_t) * mpad * cw);
+    c.q_ord.ensure(sizeof(uint32_t) * mpad * d);
+    if (mpad > c.m) {
+        pad_q_kernel<<<(unsigned)ceil_div(mpad - c.m, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(),
+                                                                          c.m, mpad, cw, d);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    const int64_t g0 = j_begin >> 5, g1 = ceil_div(j_end, 32);
+    const size_t grp_words = (size_t)c.W * 32;
+    c.tie.ensure(sizeof(uint32_t) * grp_words * (size_t)ceil_div(c.m, 32));
+    SKY_CUDA(cudaMemsetAsync(c.tie.as<uint32_t>() + g0 * grp_words, 0, sizeof(uint32_t) * grp_words * (g1 - g0), st));
+    switch (d) {
+        case 1: launch_a<1>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 2: launch_a<2>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 3: launch_a<3>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 4: launch_a<4>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 5: launch_a<5>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 6: launch_a<6>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 7: launch_a<7>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 8: launch_a<8>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 9: launch_a<9>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 10: launch_a<10>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 11: launch_a<11>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 12: launch_a<12>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 13: launch_b<13>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 14: launch_b<14>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 15: launch_b<15>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        case 16: launch_b<16>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+        default: throw Error{1, "d must be in [1, 16]"};
+    }
+}
+
+}  // namespace sky

@@ -1,0 +1,247 @@
+// prep.cu — K0 (validate + canonicalise + order-preserving keys), the key-sum order of Λ2, and
+// K2 (per-dimension monotone 15-bit codes), plus the S+ gathers after the prefilter.
+//
+// Paper: Alg. 3 line 2 (L315) builds "quad tree T over S+(P)" with global pivots (median, quartiles,
+// octiles: L338, L348-356; Fig. 3): every point gets, per dimension, its bin among
+// statically defined global thresholds, and two points are compared through their bins (Eq. 1,
+// L1312) before any exact dominance test.  This repo keeps that idea — global, monotone,
+// per-dimension bins — but with 2^15 bins per dimension (dense ranks, made coarser only when a
+// dimension has more than 2^15 distinct values), so that the bin comparison is exact for any
+// dimension with <= 2^15 distinct values and almost always decisive otherwise.
+#include "ctx.cuh"
+
+namespace sky {
+namespace {
+
+// Order-preserving image of a binary32 (after -0 -> +0): a < b  <=>  ord(a) < ord(b) for non-NaN.
+__device__ __forceinline__ uint32_t ord_key(float x) {
+    uint32_t b = __float_as_uint(x);
+    if ((b & 0x7fffffffu) == 0) b = 0;             // -0 == +0 (reading Q11)
+    return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+
+// K0: one thread per point.
+__global__ void k0_canon_kernel(const float *__restrict__ pts, int64_t n, int d, uint32_t *__restrict__ ord,
+                                uint64_t *__restrict__ keysum, uint32_t *__restrict__ perm,
+                                uint64_t *__restrict__ comp_keys, uint32_t *__restrict__ comp_vals,
+                                uint32_t *__restrict__ nanflag) {
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    uint64_t s = 0;
+    bool nan = false;
+    for (int i = 0; i < d; i++) {
+        const float x = pts[p * d + i];
+        nan |= (x != x);
+        const uint32_t o = ord_key(x);
+        ord[p * d + i] = o;
+        s += o;                                      // exact: d * 2^32 < 2^37 (Λ2)
+        comp_keys[(int64_t)i * n + p] = ((uint64_t)i << 32) | o;
+        comp_vals[(int64_t)i * n + p] = (uint32_t)p;
+    }
+    keysum[p] = s;
+    perm[p] = (uint32_t)p;
+    if (nan) atomicOr(nanflag, 1u);
+}
+
+// flags[t] = 1 iff t starts a run of equal (dim, key) in the per-dimension sorted order.
+__global__ void k2_flags_kernel(const uint64_t *__restrict__ comp_keys, int64_t n, int64_t total,
+                                uint32_t *__restrict__ flags) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= total) return;
+    flags[t] = (t % n == 0 || comp_keys[t] != comp_keys[t - 1]) ? 1u : 0u;
+}
+
+// R[dim] = number of distinct values of dimension dim.
+__global__ void k2_distinct_kernel(const uint32_t *__restrict__ ex, const uint32_t *__restrict__ flags,
+                                   int64_t n, int d, uint32_t *__restrict__ R) {
+    const int i = threadIdx.x;
+    if (i >= d) return;
+    const int64_t a = (int64_t)i * n, b = (int64_t)(i + 1) * n - 1;
+    R[i] = (ex[b] + flags[b]) - (ex[a] + flags[a]) + 1u;
+}
+
+// code = dense rank if the dimension has <= 2^15 distinct values, else floor(rank * 2^15 / R):
+// monotone in the value and equal for equal values (Λ3); injective iff R <= 2^15.
+__global__ void k2_codes_kernel(const uint32_t *__restrict__ ex, const uint32_t *__restrict__ flags,
+                                const uint32_t *__restrict__ comp_vals, const uint32_t *__restrict__ R,
+                                int64_t n, int64_t total, int dp, uint16_t *__restrict__ codes) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= total) return;
+    const int dim = (int)(t / n);
+    const int64_t a = (int64_t)dim * n;
+    const uint32_t rank = (ex[t] + flags[t]) - (ex[a] + flags[a]);
+    const uint32_t r = R[dim];
+    const uint32_t code = r <= kCodeLevels ? rank : (uint32_t)(((uint64_t)rank * kCodeLevels) / r);
+    codes[(int64_t)comp_vals[t] * dp + dim] = (uint16_t)code;
+}
+
+// Padding dimensions d..dp-1 carry code 1 on the competitor side (the task side zeroes them).
+__global__ void k2_pad_kernel(int64_t n, int d, int dp, uint16_t *__restrict__ codes) {
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    for (int i = d; i < dp; i++) codes[p * dp + i] = 1;
+}
+
+__global__ void gather_sorted_kernel(const uint32_t *__restrict__ perm, const uint32_t *__restrict__ codes_id,
+                                     const uint32_t *__restrict__ ord, int64_t n, int d, int cw,
+                                     uint32_t *__restrict__ codes_sorted, uint32_t *__restrict__ ord_sorted) {
+    const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    const int64_t id = perm[s];
+    for (int k = 0; k < cw; k++) codes_sorted[s * cw + k] = codes_id[id * cw + k];
+    for (int i = 0; i < d; i++) ord_sorted[s * d + i] = ord[id * d + i];
+}
+
+__global__ void ext_scatter_kernel(const uint32_t *__restrict__ perm, const uint8_t *__restrict__ ext_sorted,
+                                   int64_t n, uint32_t *__restrict__ ext_id_flag, uint32_t *__restrict__ key_flag) {
+    const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    const uint32_t f = ext_sorted[s] ? 1u : 0u;
+    ext_id_flag[perm[s]] = f;
+    key_flag[s] = f;
+}
+
+__global__ void ext_build_id_kernel(const uint32_t *__restrict__ ext_id_flag, const uint32_t *__restrict__ ext_idx,
+                                    const uint32_t *__restrict__ codes_id, const uint32_t *__restrict__ ord,
+                                    int64_t n, int d, int cw, int32_t *__restrict__ ext_ids,
+                                    uint32_t *__restrict__ p_codes, uint32_t *__restrict__ p_ord) {
+    const int64_t id = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (id >= n || !ext_id_flag[id]) return;
+    const int64_t j = ext_idx[id];
+    ext_ids[j] = (int32_t)id;
+    for (int k = 0; k < cw; k++) p_codes[j * cw + k] = codes_id[id * cw + k];
+    for (int i = 0; i < d; i++) p_ord[j * d + i] = ord[id * d + i];
+}
+
+__global__ void ext_build_key_kernel(const uint32_t *__restrict__ key_flag, const uint32_t *__restrict__ key_idx,
+                                     const uint32_t *__restrict__ codes_sorted, const uint32_t *__restrict__ ord_sorted,
+                                     int64_t n, int d, int cw, uint32_t *__restrict__ q_codes,
+                                     uint32_t *__restrict__ q_ord) {
+    const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n || !key_flag[s]) return;
+    const int64_t jk = key_idx[s];
+    for (int k = 0; k < cw; k++) q_codes[jk * cw + k] = codes_sorted[s * cw + k];
+    for (int i = 0; i < d; i++) q_ord[jk * d + i] = ord_sorted[s * d + i];
+}
+
+inline unsigned blocks_for(int64_t n, int t) { return (unsigned)ceil_div(n > 0 ? n : 1, t); }
+
+}  // namespace
+
+void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) {
+    c.n = n;
+    c.d = d;
+    c.dp = dpad_of(d);
+    c.W = words_per_row(d);
+    c.prepared = false;
+    c.ext_ready = false;
+    c.m = 0;
+    const int64_t nd = n * d;
+    const int cw = c.dp / 2;  // 32-bit code words per point
+    c.ord.ensure(sizeof(uint32_t) * nd);
+    c.keysum.ensure(sizeof(uint64_t) * n);
+    c.perm.ensure(sizeof(uint32_t) * n);
+    c.comp_keys.ensure(sizeof(uint64_t) * nd);
+    c.comp_vals.ensure(sizeof(uint32_t) * nd);
+    c.keys_alt.ensure(sizeof(uint64_t) * nd);
+    c.vals_alt.ensure(sizeof(uint32_t) * nd);
+    c.counts.ensure(sizeof(uint32_t) * radix_scratch_counts(nd));
+    c.scan_tmp.ensure(scan_tmp_bytes((int64_t)radix_scratch_counts(nd) > nd ? (int64_t)radix_scratch_counts(nd) : nd));
+    c.flags.ensure(sizeof(uint32_t) * nd);
+    c.scanned.ensure(sizeof(uint32_t) * nd);
+    c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
+    c.nanflag.ensure(sizeof(uint32_t));
+    c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
+    c.codes_sorted.ensure(sizeof(uint16_t) * n * c.dp);
+    c.ord_sorted.ensure(sizeof(uint32_t) * nd);
+
+    SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
+    k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, c.ord.as<uint32_t>(), c.keysum.as<uint64_t>(),
+                                                        c.perm.as<uint32_t>(), c.comp_keys.as<uint64_t>(),
+                                                        c.comp_vals.as<uint32_t>(), c.nanflag.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    uint32_t nan = 0;
+    SKY_CUDA(cudaMemcpyAsync(&nan, c.nanflag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    SKY_CUDA(cudaStreamSynchronize(st));
+    if (nan) throw Error{2, "NaN in input points"};
+
+    // Λ2 order: sum of order-preserving keys (< 2^36 for d <= 16), stable by id.
+    radix_sort_u64(c.keysum.as<uint64_t>(), c.perm.as<uint32_t>(), n, 36, c.keys_alt.as<uint64_t>(),
+                   c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
+    // K2: per-dimension sort of (dim, key) -> dense ranks -> codes.
+    radix_sort_u64(c.comp_keys.as<uint64_t>(), c.comp_vals.as<uint32_t>(), nd, 36, c.keys_alt.as<uint64_t>(),
+                   c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
+    k2_flags_kernel<<<blocks_for(nd, 256), 256, 0, st>>>(c.comp_keys.as<uint64_t>(), n, nd, c.flags.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    exclusive_scan_u32(c.flags.as<uint32_t>(), c.scanned.as<uint32_t>(), nd, c.scan_tmp.p, st, c.L);
+    k2_distinct_kernel<<<1, 32, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(), n, d, c.rbuf.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    k2_codes_kernel<<<blocks_for(nd, 256), 256, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(),
+                                                         c.comp_vals.as<uint32_t>(), c.rbuf.as<uint32_t>(), n, nd,
+                                                         c.dp, c.codes_id.as<uint16_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    if (c.dp > d) {
+        k2_pad_kernel<<<blocks_for(n, 256), 256, 0, st>>>(n, d, c.dp, c.codes_id.as<uint16_t>());
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    SKY_CUDA(cudaMemcpyAsync(c.R, c.rbuf.p, sizeof(uint32_t) * d, cudaMemcpyDeviceToHost, st));
+    gather_sorted_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
+                                                             c.ord.as<uint32_t>(), n, d, cw,
+                                                             c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    SKY_CUDA(cudaStreamSynchronize(st));
+    c.exact_mask = 0;
+    for (int i = 0; i < d; i++)
+        if (c.R[i] <= kCodeLevels) c.exact_mask |= 1u << i;
+    c.prepared = true;
+}
+
+void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
+    if (!c.prepared) throw Error{1, "skycube_dev_set_ext before skycube_dev_prepare"};
+    const int64_t n = c.n;
+    const int d = c.d;
+    const int cw = c.dp / 2;
+    c.ext_id_flag.ensure(sizeof(uint32_t) * n);
+    c.ext_idx.ensure(sizeof(uint32_t) * n);
+    c.key_flag.ensure(sizeof(uint32_t) * n);
+    c.key_idx.ensure(sizeof(uint32_t) * n);
+    c.scan_tmp.ensure(scan_tmp_bytes(n));
+    ext_scatter_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.perm.as<uint32_t>(), d_ext_sorted, n,
+                                                           c.ext_id_flag.as<uint32_t>(), c.key_flag.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    exclusive_scan_u32(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(), n, c.scan_tmp.p, st, c.L);
+    exclusive_scan_u32(c.key_flag.as<uint32_t>(), c.key_idx.as<uint32_t>(), n, c.scan_tmp.p, st, c.L);
+    uint32_t last[2];
+    SKY_CUDA(cudaMemcpyAsync(&last[0], c.ext_idx.as<uint32_t>() + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    SKY_CUDA(cudaMemcpyAsync(&last[1], c.ext_id_flag.as<uint32_t>() + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    SKY_CUDA(cudaStreamSynchronize(st));
+    const int64_t m = (int64_t)last[0] + last[1];
+    c.m = m;
+    const int64_t mm = m > 0 ? m : 1;
+    c.ext_ids.ensure(sizeof(int32_t) * mm);
+    c.p_codes.ensure(sizeof(uint16_t) * (mm + 32) * c.dp);
+    c.p_ord.ensure(sizeof(uint32_t) * mm * d);
+    c.q_codes.ensure(sizeof(uint16_t) * (mm + 1024) * c.dp);
+    c.q_ord.ensure(sizeof(uint32_t) * mm * d);
+    ext_build_id_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(),
+                                                            c.codes_id.as<uint32_t>(), c.ord.as<uint32_t>(), n, d, cw,
+                                                            c.ext_ids.as<int32_t>(), c.p_codes.as<uint32_t>(),
+                                                            c.p_ord.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    ext_build_key_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.key_flag.as<uint32_t>(), c.key_idx.as<uint32_t>(),
+                                                             c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>(),
+                                                             n, d, cw, c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    c.ext_ready = true;
+}
+
+}  // namespace sky

@@ -1,0 +1,151 @@
+"""Bit-exact parity of the CUDA path (through the C-ABI) against the CPU oracle — needs a B200."""
+from __future__ import annotations
+
+import json
+import os
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+import paper_conf_sigmod_boghcsa17_b200 as sky
+from pins import fig3_string, members
+
+pytestmark = pytest.mark.gpu
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "flights.json")))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    sky.lib()
+
+
+def gpu(x, **kw):
+    return sky.skycube_build(x, ext_membership=True, **kw)
+
+
+def check_against_oracle(x, res, ext=True):
+    n, d = x.shape
+    want_rows, want_ext = oracle.rows_b(x, with_ext=True)
+    assert res["rows"].shape == want_rows.shape
+    bad = np.nonzero((res["rows"] != want_rows).any(axis=1))[0]
+    assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
+    want_ext_ids = np.nonzero(oracle.ext_full(x))[0]
+    assert np.array_equal(res["ext_ids"], want_ext_ids)
+    if ext:
+        # B_{p in S+} rows are only produced for S+ points (others are zero by construction)
+        er = res["ext_rows"]
+        assert np.array_equal(er[want_ext_ids], want_ext[want_ext_ids])
+    off, ids = oracle.lattice(want_rows, d)
+    assert np.array_equal(res["offsets"], off)
+    assert np.array_equal(res["ids"], ids)
+
+
+def test_flights_table1():
+    x = np.array(GOLD["points"], np.float32)
+    r = gpu(x)
+    for delta_s, ids in GOLD["lattice"].items():
+        assert members(r["rows"], int(delta_s)) == ids
+    assert r["offsets"].tolist() == [0, 0, 1, 2, 5, 6, 9, 12, 16]
+    assert r["ext_ids"].tolist() == [0, 1, 2, 3, 4]
+    for p in range(5):
+        assert fig3_string(r["rows"], p, 3, negate=True) == GOLD["fig3_not_in_S"][p]
+        assert fig3_string(r["ext_rows"], p, 3, negate=True) == GOLD["fig3_not_in_Sp"][p]
+
+
+def test_c1_all_15_cuboids_vs_oracle_a():
+    x = datagen.config("C1").data()
+    r = gpu(x)
+    rows = oracle.rows_a(x, with_ext=False)
+    assert np.array_equal(r["rows"], rows)
+    off, ids = oracle.lattice(rows, 4)
+    assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)
+
+
+@pytest.mark.parametrize("d", list(range(1, 17)))
+def test_every_d_tie_heavy(d):
+    x = datagen.small_int_grid(150 if d < 14 else 90, d, 3, 100 + d)
+    check_against_oracle(x, gpu(x))
+
+
+@pytest.mark.parametrize("d", list(range(1, 17)))
+def test_every_d_anticorrelated(d):
+    x = datagen.generate("A", 300 if d < 14 else 160, d, 200 + d)
+    check_against_oracle(x, gpu(x))
+
+
+@pytest.mark.parametrize("dist,n,d,seed", [
+    ("A", 4000, 12, 1),     # ~30 competitor tiles, ragged tail
+    ("I", 6000, 8, 2),
+    ("C", 5000, 12, 3),
+    ("ct", 3000, 10, 4),    # heavy ties, exact codes
+    ("A", 1500, 16, 5),     # design B
+    ("A", 2500, 13, 6),
+    ("I", 3000, 5, 7),
+])
+def test_medium_vs_oracle(dist, n, d, seed):
+    x = datagen.generate(dist, n, d, seed)
+    check_against_oracle(x, gpu(x))
+
+
+def test_inexact_codes_refinement():
+    # > 2^15 distinct values per dimension forces non-injective codes (refinement path), with
+    # clustered values so that many pairs share a code.
+    rng = np.random.default_rng(5)
+    n, d = 40000, 4
+    base = rng.integers(0, 1 << 20, size=(n, d)).astype(np.float32)
+    x = np.ascontiguousarray(base)
+    r = gpu(x)
+    pids = rng.choice(n, 300, replace=False)
+    want = oracle.rows_b(x, pids)
+    assert np.array_equal(r["rows"][pids], want)
+
+
+def test_edge_cases():
+    # n = 1
+    r = gpu(np.array([[0.5, 0.25, 0.75]], np.float32))
+    assert r["rows"][0, 0] == 0xFE and r["ext_ids"].tolist() == [0]
+    # all identical
+    r = gpu(np.ones((70, 5), np.float32))
+    assert (r["rows"][:, 0] == 0xFFFFFFFE).all()
+    # chain / antichain
+    x = datagen.chain(100, 6)
+    check_against_oracle(x, gpu(x))
+    x = datagen.antichain2d(77)
+    check_against_oracle(x, gpu(x))
+    # -0 / +0 / inf
+    x = np.array([[-np.inf, 1.0], [0.0, -0.0], [-0.0, 0.0], [np.inf, np.inf]], np.float32)
+    check_against_oracle(x, gpu(x))
+    # n = 0
+    r = gpu(np.zeros((0, 7), np.float32))
+    assert r["rows"].shape == (0, 4) and r["offsets"].tolist() == [0] * 129
+
+
+def test_nan_rejected():
+    x = np.ones((10, 3), np.float32)
+    x[4, 1] = np.nan
+    with pytest.raises(sky.SkycubeError) as e:
+        gpu(x)
+    assert e.value.status == sky.ENAN
+
+
+def test_no_lists_flag_and_repeat_calls():
+    x = datagen.generate("A", 2000, 9, 9)
+    a = sky.skycube_build(x, lists=False)
+    b = sky.skycube_build(x)
+    assert "offsets" not in a and np.array_equal(a["rows"], b["rows"])
+    c = sky.skycube_build(x)
+    assert np.array_equal(b["ids"], c["ids"])
+
+
+def test_row_permutation_invariance():
+    x = datagen.generate("I", 3000, 7, 11)
+    perm = np.random.default_rng(0).permutation(3000)
+    a = gpu(x)["rows"]
+    b = gpu(x[perm])["rows"]
+    assert np.array_equal(a[perm], b)
