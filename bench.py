@@ -42,9 +42,11 @@ def algorithmic_ops_per_pair(d: int) -> int:
 
 
 def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
-    """ALU pipe peak (B300_MICROARCH.md: IADD3/LOP3/SHF/PRMT on the alu pipe, rt = 2 cycles per warp
-    instruction per SMSP -> 16 lanes/SMSP, 64 lanes/SM per clock)."""
-    return sms * 64 * sm_mhz * 1e6
+    """Integer issue peak (DESIGN.md §Roofline): each SMSP issues at most one warp instruction per clock;
+    integer work runs on the ALU pipe (IADD3/LOP3/SHF/PRMT, 16 lanes/SMSP) and on the FMA pipe
+    (IMAD/IMAD.IADD, 16 lanes/SMSP) (B300_MICROARCH.md "Pipe rates"), so 4 x 32 = 128 integer lane-ops
+    per SM per clock."""
+    return sms * 128 * sm_mhz * 1e6
 
 
 def env_rank():
@@ -268,7 +270,8 @@ def run_ours(args):
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
                      "frac": achieved / peak, "traffic": None,
                      "kernel": "k3_mdmc", "ops_per_pair": algorithmic_ops_per_pair(d),
-                     "peak_basis": f"148 SM x 64 ALU lanes x {sm_mhz:.0f} MHz (median SM clock under load)"},
+                     "peak_basis": f"148 SM x 128 integer lanes/clk (ALU+FMA pipes, 1 warp-inst/SMSP/clk) x {sm_mhz:.0f} MHz "
+                                   f"(median SM clock under load)"},
         "clocks": clocks,
     }
     if e2e is not None:

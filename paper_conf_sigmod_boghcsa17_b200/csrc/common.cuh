@@ -43,6 +43,7 @@ struct Error {
 inline uint32_t words_per_row(int d) { return d >= 5 ? (1u << (d - 5)) : 1u; }
 inline int dpad_of(int d) { return ((d + 3) / 4) * 4; }  // codes padded to groups of 4 dims
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+__device__ __forceinline__ int64_t ceil_div_dev(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 // ------------------------------------------------------------------------------ sort / scan API
 // Stable LSD radix sort of (key, value) pairs on the low `bits` bits of the 64-bit keys.

@@ -25,6 +25,7 @@
 //   design B (d > 12): one warp per task (PPW tasks per warp), lanes stride over q; the 2^d-bit state
 //     (8 KB at d = 16) is shared by the warp; misses expand with shared atomics.
 #include "ctx.cuh"
+#include "tile_stream.cuh"
 
 namespace sky {
 namespace {
@@ -79,21 +80,68 @@ __device__ __forceinline__ void refine_exact(uint32_t U, const uint32_t *__restr
 // ==================================================================================== design A
 constexpr int kAWarps = 4;
 constexpr int kATQ = 128;  // competitors per shared-memory tile
+constexpr int kAU = 8;     // competitors per inner iteration (independent chains for ILP)
+constexpr int kAStages = 3;  // TMA ring depth
+
+// The rare miss path for one (p, q) pair (Alg. 3 lines 10-12).  Returns true if a tie row was written.
+template <int D>
+__device__ __forceinline__ bool mdmc_miss(uint32_t *st, const uint32_t *pH, const uint32_t *qw, uint32_t M,
+                                          uint32_t inexact, const uint32_t *__restrict__ qo,
+                                          const uint32_t *__restrict__ po, uint32_t *tr) {
+    using G = Geo<D>;
+    uint32_t lt[G::CW];
+#pragma unroll
+    for (int k = 0; k < G::CW; k++) lt[k] = pH[k] - qw[k] - 0x00010001u;  // guard <=> code(q) < code(p)
+    uint32_t S = gather_mask<G::NG>(lt);
+    uint32_t L = M;
+    const uint32_t U = M & ~S & inexact;
+    if (U) refine_exact(U, qo, po, L, S);
+    if (S == 0) return false;                                         // q is nowhere better than p
+    if (L != M && ((st[(L >> 5) * 32] >> (L & 31)) & 1u)) return false;
+    {   // B_{p notin S+} |= sub(S)   (strict dominance propagates to all submasks, L330)
+        const uint32_t sh = S >> 5, bits = sub5(S & 31u);
+        uint32_t w = 0;
+        do {
+            st[w * 32] |= bits;
+            w = (w - sh) & sh;
+        } while (w);
+    }
+    if (L == S) return false;
+    // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}  (reading Q3)
+    const uint32_t E = L & ~S;
+    const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
+    uint32_t w = 0;
+    do {
+        tr[w * 32] |= (w & ~eh) ? lb : (lb & ~eb);
+        w = (w - lh) & lh;
+    } while (w);
+    return true;
+}
 
 template <int D>
-__global__ void __launch_bounds__(kAWarps * 32) k3_mdmc_a_kernel(
+__global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ q_codes,
     const uint32_t *__restrict__ q_ord, int64_t ntiles_q, int64_t j_begin, int64_t j_end, uint32_t inexact,
     uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
     using G = Geo<D>;
-    extern __shared__ uint32_t smem[];
-    uint32_t *qs = smem;                                            // [kATQ][CW]
+    extern __shared__ __align__(128) uint32_t smem[];
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);             // full[kAStages], empty[kAStages]
+    const TileRing<kAStages> ring{bars, bars + kAStages, smem + 4 * kAStages, (uint32_t)(kATQ * G::CW)};
+    uint32_t *stbase = smem + 4 * kAStages + kAStages * kATQ * G::CW;  // [kAWarps][WB][32]
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    uint32_t *st = smem + kATQ * G::CW + warp * G::WB * 32 + lane;  // word w of this task: st[w * 32]
+    uint32_t *st = stbase + warp * G::WB * 32 + lane;                // word w of this task: st[w * 32]
     const int64_t j = j_begin + (int64_t)blockIdx.x * (kAWarps * 32) + warp * 32 + lane;
     const bool active = j < j_end;
     const int64_t grp = j >> 5;
+    uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
 
+    if (threadIdx.x == 0) ring.init(kAWarps);
+    if (warp == kAWarps) {  // producer warp: one elected lane streams competitor tiles with TMA
+        __syncthreads();
+        if (lane == 0)
+            for (int64_t t = 0; t < ntiles_q; t++) ring.issue(q_codes, t);
+        return;
+    }
     uint32_t pH[G::CW];
 #pragma unroll
     for (int k = 0; k < G::CW; k++) {
@@ -105,68 +153,47 @@ __global__ void __launch_bounds__(kAWarps * 32) k3_mdmc_a_kernel(
 #pragma unroll 4
     for (int w = 0; w < G::WB; w++) st[w * 32] = w == 0 ? 1u : 0u;  // bit 0 (empty subspace) preset
     bool had_tie = false;
+    __syncthreads();
+    const char *stc = reinterpret_cast<const char *>(st);
 
     for (int64_t tq = 0; tq < ntiles_q; tq++) {
-        __syncthreads();
-        {
-            const uint4 *src = reinterpret_cast<const uint4 *>(q_codes + tq * kATQ * G::CW);
-            uint4 *dst = reinterpret_cast<uint4 *>(qs);
-            for (int i = threadIdx.x; i < kATQ * G::CW / 4; i += kAWarps * 32) dst[i] = src[i];
-        }
-        __syncthreads();
-        if (!active) continue;
-#pragma unroll 2
-        for (int t = 0; t < kATQ; t++) {
-            const uint32_t *qw = qs + t * G::CW;
-            uint32_t le[G::CW];
+        ring.wait(tq);
+        const uint32_t *qs = ring.stage(tq);
+        if (active) {
+#pragma unroll 1
+            for (int t = 0; t < kATQ; t += kAU) {
+                uint32_t M[kAU], wd[kAU];
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) le[k] = pH[k] - qw[k];  // guard <=> code(q) <= code(p)
-            const uint32_t M = gather_mask<G::NG>(le);
-            const uint32_t word = st[(M >> 5) * 32];
-            if ((word >> (M & 31)) & 1u) continue;                     // Λ4: nothing new from q
-            // ---- miss: exact masks, then Alg. 3 line 12
-            uint32_t lt[G::CW];
+                for (int u = 0; u < kAU; u++) {
+                    const uint32_t *qw = qs + (t + u) * G::CW;
+                    uint32_t le[G::CW];
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) lt[k] = pH[k] - qw[k] - 0x00010001u;  // guard <=> code(q) < code(p)
-            uint32_t S = gather_mask<G::NG>(lt);
-            uint32_t L = M;
-            const uint32_t U = M & ~S & inexact;
-            if (U) {
-                const int64_t q = tq * kATQ + t;
-                refine_exact(U, q_ord + q * D, p_ord + j * D, L, S);
-            }
-            if (S == 0) continue;                                      // q is nowhere better than p
-            if (L != M && ((st[(L >> 5) * 32] >> (L & 31)) & 1u)) continue;
-            {   // B_{p notin S+} |= sub(S)   (strict dominance propagates to all submasks, L330)
-                const uint32_t sh = S >> 5, bits = sub5(S & 31u);
-                uint32_t w = 0;
-                do {
-                    st[w * 32] |= bits;
-                    w = (w - sh) & sh;
-                } while (w);
-            }
-            if (L != S) {  // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}
-                const uint32_t E = L & ~S;
-                const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
-                uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
-                uint32_t w = 0;
-                do {
-                    const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
-                    tr[w * 32] |= bits;
-                    w = (w - lh) & lh;
-                } while (w);
-                had_tie = true;
+                    for (int k = 0; k < G::CW; k++) le[k] = pH[k] - qw[k];  // guard <=> code(q) <= code(p)
+                    M[u] = gather_mask<G::NG>(le);
+                }
+#pragma unroll
+                for (int u = 0; u < kAU; u++) wd[u] = *reinterpret_cast<const uint32_t *>(stc + ((M[u] >> 5) << 7));
+                uint32_t hit = 0xffffffffu;
+#pragma unroll
+                for (int u = 0; u < kAU; u++) hit &= __funnelshift_r(wd[u], wd[u], M[u]);  // bit M of B_{p notin S+}
+                if (hit & 1u) continue;                                   // Λ4: none of the kAU competitors adds anything
+#pragma unroll
+                for (int u = 0; u < kAU; u++) {
+                    if ((st[(M[u] >> 5) * 32] >> (M[u] & 31)) & 1u) continue;
+                    const int64_t q = tq * kATQ + t + u;
+                    had_tie |= mdmc_miss<D>(st, pH, qs + (t + u) * G::CW, M[u], inexact, q_ord + q * D, p_ord + j * D, tr);
+                }
             }
         }
+        __syncwarp();
+        if (lane == 0) ring.release(tq);
     }
     if (!active) return;
-    const bool any_tie = __any_sync(__activemask(), had_tie);
     uint32_t *out = rows32 + grp * (G::WB * 32) + lane;
-    const uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
 #pragma unroll 4
     for (int w = 0; w < G::WB; w++) {
         uint32_t v = st[w * 32];
-        if (any_tie && had_tie) v |= tr[w * 32];
+        if (had_tie) v |= tr[w * 32];
         uint32_t row = ~v & G::kRowMask;
         if (w == 0) row &= ~1u;
         out[w * 32] = row;
@@ -296,11 +323,11 @@ __global__ void __launch_bounds__(kBWarps * 32) k3_mdmc_b_kernel(
 template <int D>
 void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
-    const size_t smem = sizeof(uint32_t) * ((size_t)kATQ * G::CW + (size_t)kAWarps * G::WB * 32);
+    const size_t smem = sizeof(uint32_t) * (4 * kAStages + kAStages * (size_t)kATQ * G::CW + (size_t)kAWarps * G::WB * 32);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_a_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int64_t ntq = ceil_div(c.m, kATQ);
     const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, kAWarps * 32);
-    k3_mdmc_a_kernel<D><<<blocks, kAWarps * 32, smem, st>>>(
+    k3_mdmc_a_kernel<D><<<blocks, (kAWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(), ntq,
         j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
     c.L.count++;

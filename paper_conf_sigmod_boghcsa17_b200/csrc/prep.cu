@@ -86,7 +86,11 @@ __global__ void gather_sorted_kernel(const uint32_t *__restrict__ perm, const ui
                                      const uint32_t *__restrict__ ord, int64_t n, int d, int cw,
                                      uint32_t *__restrict__ codes_sorted, uint32_t *__restrict__ ord_sorted) {
     const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (s >= n) return;
+    if (s >= n) {  // padding up to whole K1 tiles: codes that never pass the q <= p test
+        if (s < ((n + 255) / 256) * 256)
+            for (int k = 0; k < cw; k++) codes_sorted[s * cw + k] = 0x7fff7fffu;
+        return;
+    }
     const int64_t id = perm[s];
     for (int k = 0; k < cw; k++) codes_sorted[s * cw + k] = codes_id[id * cw + k];
     for (int i = 0; i < d; i++) ord_sorted[s * d + i] = ord[id * d + i];
@@ -152,7 +156,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
     c.nanflag.ensure(sizeof(uint32_t));
     c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
-    c.codes_sorted.ensure(sizeof(uint16_t) * n * c.dp);
+    c.codes_sorted.ensure(sizeof(uint16_t) * (n + 256) * c.dp);
     c.ord_sorted.ensure(sizeof(uint32_t) * nd);
 
     SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
@@ -190,7 +194,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
         SKY_LAUNCH_CHECK();
     }
     SKY_CUDA(cudaMemcpyAsync(c.R, c.rbuf.p, sizeof(uint32_t) * d, cudaMemcpyDeviceToHost, st));
-    gather_sorted_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
+    gather_sorted_kernel<<<blocks_for(n, 256) + 1, 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
                                                              c.ord.as<uint32_t>(), n, d, cw,
                                                              c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>());
     c.L.count++;
