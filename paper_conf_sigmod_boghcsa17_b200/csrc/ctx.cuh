@@ -82,5 +82,6 @@ void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *
                      cudaStream_t st);
 
 constexpr int kPrefilterTile = 256;  // sorted positions per K1 block
+constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
 
 }  // namespace sky

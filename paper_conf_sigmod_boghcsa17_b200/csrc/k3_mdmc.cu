@@ -22,8 +22,9 @@
 //   design A (d <= 12): one thread per task p, a warp = 32 tasks, every competitor q is read once per
 //     CTA from shared memory as a broadcast; B_{p notin S+} lives in shared memory as [word][lane]
 //     (bank = lane, conflict-free probes).  2^d/8 bytes per task.
-//   design B (d > 12): one warp per task (PPW tasks per warp), lanes stride over q; the 2^d-bit state
-//     (8 KB at d = 16) is shared by the warp; misses expand with shared atomics.
+//   design B (d > 12): a CTA holds the states of NT tasks (192 KB in total, 8 KB per task at d = 16);
+//     each lane holds one competitor in registers and runs it against all NT tasks (task codes are
+//     broadcasts); misses expand with shared-memory atomics.
 #include "ctx.cuh"
 #include "tile_stream.cuh"
 
@@ -84,6 +85,7 @@ constexpr int kAU = 8;     // competitors per inner iteration (independent chain
 constexpr int kAStages = 3;  // TMA ring depth
 
 // The rare miss path for one (p, q) pair (Alg. 3 lines 10-12).  Returns true if a tie row was written.
+// `tr` points at word 0 of the task's tie row, stride 32 words: shared memory (TIES layout) or global.
 template <int D>
 __device__ __forceinline__ bool mdmc_miss(uint32_t *st, const uint32_t *pH, const uint32_t *qw, uint32_t M,
                                           uint32_t inexact, const uint32_t *__restrict__ qo,
@@ -98,7 +100,7 @@ __device__ __forceinline__ bool mdmc_miss(uint32_t *st, const uint32_t *pH, cons
     if (U) refine_exact(U, qo, po, L, S);
     if (S == 0) return false;                                         // q is nowhere better than p
     if (L != M && ((st[(L >> 5) * 32] >> (L & 31)) & 1u)) return false;
-    {   // B_{p notin S+} |= sub(S)   (strict dominance propagates to all submasks, L330)
+    if (!((st[(S >> 5) * 32] >> (S & 31)) & 1u)) {  // B_{p notin S+} |= sub(S) (strict dominance propagates)
         const uint32_t sh = S >> 5, bits = sub5(S & 31u);
         uint32_t w = 0;
         do {
@@ -118,7 +120,7 @@ __device__ __forceinline__ bool mdmc_miss(uint32_t *st, const uint32_t *pH, cons
     return true;
 }
 
-template <int D>
+template <int D, bool TIES>
 __global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ q_codes,
     const uint32_t *__restrict__ q_ord, int64_t ntiles_q, int64_t j_begin, int64_t j_end, uint32_t inexact,
@@ -133,7 +135,8 @@ __global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
     const int64_t j = j_begin + (int64_t)blockIdx.x * (kAWarps * 32) + warp * 32 + lane;
     const bool active = j < j_end;
     const int64_t grp = j >> 5;
-    uint32_t *tr = tie32 + grp * (G::WB * 32) + lane;
+    // TIES: the tie part of B_{p notin S} also lives in shared memory (tie-heavy / low-d inputs)
+    uint32_t *tr = TIES ? stbase + (kAWarps + warp) * G::WB * 32 + lane : tie32 + grp * (G::WB * 32) + lane;
 
     if (threadIdx.x == 0) ring.init(kAWarps);
     if (warp == kAWarps) {  // producer warp: one elected lane streams competitor tiles with TMA
@@ -151,7 +154,10 @@ __global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
         pH[k] = w | kGuard;
     }
 #pragma unroll 4
-    for (int w = 0; w < G::WB; w++) st[w * 32] = w == 0 ? 1u : 0u;  // bit 0 (empty subspace) preset
+    for (int w = 0; w < G::WB; w++) {
+        st[w * 32] = w == 0 ? 1u : 0u;  // bit 0 (empty subspace) preset
+        if (TIES) tr[w * 32] = 0u;
+    }
     bool had_tie = false;
     __syncthreads();
     const char *stc = reinterpret_cast<const char *>(st);
@@ -193,7 +199,7 @@ __global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
 #pragma unroll 4
     for (int w = 0; w < G::WB; w++) {
         uint32_t v = st[w * 32];
-        if (had_tie) v |= tr[w * 32];
+        if (TIES || had_tie) v |= tr[w * 32];
         uint32_t row = ~v & G::kRowMask;
         if (w == 0) row &= ~1u;
         out[w * 32] = row;
@@ -206,142 +212,178 @@ __global__ void __launch_bounds__((kAWarps + 1) * 32) k3_mdmc_a_kernel(
 }
 
 // ==================================================================================== design B
-constexpr int kBWarps = 8;
-constexpr int kBPPW = 2;   // tasks per warp
-constexpr int kBTQ = 256;  // competitors per tile
+// d > 12: the 2^d-bit state (1-8 KB per task) is too large for one task per thread.  A CTA keeps the
+// states of NT tasks in shared memory and every consumer warp holds 32 competitors in registers (one
+// per lane, read once from the TMA-fed tile) and runs them against all NT tasks: the task's codes are
+// a shared-memory broadcast, the probe goes to the task's state (random words: some bank conflicts),
+// misses expand with shared-memory atomics (several warps may update one task's state).
+constexpr int kBWarps = 16;           // consumer warps (+1 producer warp)
+constexpr int kBTQ = kBWarps * 32;    // competitors per tile: one per consumer lane
+constexpr int kBStages = 3;
+constexpr int kBStateBytes = 160 * 1024;
+constexpr int kBTU = 4;               // tasks per inner iteration (independent chains)
 
 template <int D>
-__global__ void __launch_bounds__(kBWarps * 32) k3_mdmc_b_kernel(
+struct GeoB {
+    static constexpr int NT = kBStateBytes / (Geo<D>::WB * 4) < 256 ? kBStateBytes / (Geo<D>::WB * 4) : 256;
+};
+
+template <int D>
+__device__ __forceinline__ void mdmc_miss_b(uint32_t *st, const uint32_t *pH, const uint32_t *qw, uint32_t M,
+                                            uint32_t inexact, const uint32_t *__restrict__ qo,
+                                            const uint32_t *__restrict__ po, uint32_t *tr) {
+    using G = Geo<D>;
+    uint32_t lt[G::CW];
+#pragma unroll
+    for (int k = 0; k < G::CW; k++) lt[k] = pH[k] - qw[k] - 0x00010001u;
+    uint32_t S = gather_mask<G::NG>(lt);
+    uint32_t L = M;
+    const uint32_t U = M & ~S & inexact;
+    if (U) refine_exact(U, qo, po, L, S);
+    if (S == 0) return;
+    if (L != M && ((st[L >> 5] >> (L & 31)) & 1u)) return;
+    if (!((st[S >> 5] >> (S & 31)) & 1u)) {
+        const uint32_t sh = S >> 5, bits = sub5(S & 31u);
+        uint32_t w = 0;
+        do {
+            atomicOr(&st[w], bits);
+            w = (w - sh) & sh;
+        } while (w);
+    }
+    if (L == S) return;
+    const uint32_t E = L & ~S;
+    const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
+    uint32_t w = 0;
+    do {
+        atomicOr(&tr[w * 32], (w & ~eh) ? lb : (lb & ~eb));
+        w = (w - lh) & lh;
+    } while (w);
+}
+
+template <int D>
+__global__ void __launch_bounds__((kBWarps + 1) * 32, 1) k3_mdmc_b_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ q_codes,
     const uint32_t *__restrict__ q_ord, int64_t ntiles_q, int64_t j_begin, int64_t j_end, uint32_t inexact,
     uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
     using G = Geo<D>;
-    extern __shared__ uint32_t smem[];
-    uint32_t *qs = smem;  // [kBTQ][CW]
+    constexpr int NT = GeoB<D>::NT;
+    extern __shared__ __align__(128) uint32_t smem[];
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    const TileRing<kBStages> ring{bars, bars + kBStages, smem + 4 * kBStages, (uint32_t)(kBTQ * G::CW)};
+    uint32_t *pcs = smem + 4 * kBStages + kBStages * kBTQ * G::CW;  // [NT][CW] task codes (with guard bits)
+    uint32_t *state = pcs + NT * G::CW;                              // [NT][WB]
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    uint32_t *stw = smem + kBTQ * G::CW + warp * (kBPPW * G::WB);  // [kBPPW][WB]
-    int64_t jt[kBPPW];
-    bool act[kBPPW];
-    uint32_t pH[kBPPW][G::CW];
-#pragma unroll
-    for (int s = 0; s < kBPPW; s++) {
-        jt[s] = j_begin + ((int64_t)blockIdx.x * kBWarps + warp) * kBPPW + s;
-        act[s] = jt[s] < j_end;
-#pragma unroll
-        for (int k = 0; k < G::CW; k++) {
-            uint32_t w = act[s] ? p_codes[jt[s] * G::CW + k] : 0u;
-            if (2 * k >= D) w &= 0xffff0000u;
-            if (2 * k + 1 >= D) w &= 0x0000ffffu;
-            pH[s][k] = w | kGuard;
-        }
-    }
-    for (int w = lane; w < kBPPW * G::WB; w += 32) stw[w] = (w % G::WB) == 0 ? 1u : 0u;
-    bool had_tie[kBPPW];
-#pragma unroll
-    for (int s = 0; s < kBPPW; s++) had_tie[s] = false;
-    __syncwarp();
+    const int64_t j0 = j_begin + (int64_t)blockIdx.x * NT;
+    const int nt = (int)min((int64_t)NT, j_end - j0);
 
+    if (threadIdx.x == 0) ring.init(kBWarps);
+    for (int i = threadIdx.x; i < NT * G::CW; i += blockDim.x) {
+        const int t = i / G::CW, k = i % G::CW;
+        uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
+        if (2 * k >= D) w &= 0xffff0000u;
+        if (2 * k + 1 >= D) w &= 0x0000ffffu;
+        pcs[i] = w | kGuard;
+    }
+    for (int i = threadIdx.x; i < NT * G::WB; i += blockDim.x) state[i] = (i % G::WB) == 0 ? 1u : 0u;
+    __syncthreads();
+    if (warp == kBWarps) {  // producer warp
+        if (lane == 0)
+            for (int64_t t = 0; t < ntiles_q; t++) ring.issue(q_codes, t);
+        return;
+    }
     for (int64_t tq = 0; tq < ntiles_q; tq++) {
-        __syncthreads();
-        {
-            const uint4 *src = reinterpret_cast<const uint4 *>(q_codes + tq * kBTQ * G::CW);
-            uint4 *dst = reinterpret_cast<uint4 *>(qs);
-            for (int i = threadIdx.x; i < kBTQ * G::CW / 4; i += kBWarps * 32) dst[i] = src[i];
-        }
-        __syncthreads();
-        for (int t = lane; t < kBTQ; t += 32) {
-            uint32_t qw[G::CW];
+        ring.wait(tq);
+        uint32_t qw[G::CW];
+        const uint32_t *qsrc = ring.stage(tq) + (warp * 32 + lane) * G::CW;
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) qw[k] = qs[t * G::CW + k];
+        for (int k = 0; k < G::CW; k++) qw[k] = qsrc[k];
+        __syncwarp();
+        if (lane == 0) ring.release(tq);
+        const int64_t q = tq * kBTQ + warp * 32 + lane;
+#pragma unroll 1
+        for (int t0 = 0; t0 < nt; t0 += kBTU) {
+            uint32_t M[kBTU], wd[kBTU];
 #pragma unroll
-            for (int s = 0; s < kBPPW; s++) {
-                if (!act[s]) continue;
-                uint32_t *st = stw + s * G::WB;
+            for (int u = 0; u < kBTU; u++) {
+                const int t = min(t0 + u, nt - 1);
+                const uint32_t *ph = pcs + t * G::CW;
                 uint32_t le[G::CW];
 #pragma unroll
-                for (int k = 0; k < G::CW; k++) le[k] = pH[s][k] - qw[k];
-                const uint32_t M = gather_mask<G::NG>(le);
-                if ((st[M >> 5] >> (M & 31)) & 1u) continue;
-                uint32_t lt[G::CW];
+                for (int k = 0; k < G::CW; k++) le[k] = ph[k] - qw[k];
+                M[u] = gather_mask<G::NG>(le);
+                wd[u] = state[t * G::WB + (M[u] >> 5)];
+            }
+            uint32_t hit = 0xffffffffu;
 #pragma unroll
-                for (int k = 0; k < G::CW; k++) lt[k] = pH[s][k] - qw[k] - 0x00010001u;
-                uint32_t S = gather_mask<G::NG>(lt);
-                uint32_t L = M;
-                const uint32_t U = M & ~S & inexact;
-                if (U) {
-                    const int64_t q = tq * kBTQ + t;
-                    refine_exact(U, q_ord + q * D, p_ord + jt[s] * D, L, S);
-                }
-                if (S == 0) continue;
-                if (L != M && ((st[L >> 5] >> (L & 31)) & 1u)) continue;
-                {
-                    const uint32_t sh = S >> 5, bits = sub5(S & 31u);
-                    uint32_t w = 0;
-                    do {
-                        atomicOr(&st[w], bits);
-                        w = (w - sh) & sh;
-                    } while (w);
-                }
-                if (L != S) {
-                    const uint32_t E = L & ~S;
-                    const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
-                    uint32_t *tr = tie32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
-                    uint32_t w = 0;
-                    do {
-                        const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
-                        atomicOr(&tr[w * 32], bits);
-                        w = (w - lh) & lh;
-                    } while (w);
-                    had_tie[s] = true;
-                }
+            for (int u = 0; u < kBTU; u++) hit &= __funnelshift_r(wd[u], wd[u], M[u]);
+            if (hit & 1u) continue;
+#pragma unroll
+            for (int u = 0; u < kBTU; u++) {
+                const int t = t0 + u;
+                if (t >= nt) break;
+                uint32_t *st = state + t * G::WB;
+                if ((st[M[u] >> 5] >> (M[u] & 31)) & 1u) continue;
+                const int64_t jt = j0 + t;
+                mdmc_miss_b<D>(st, pcs + t * G::CW, qw, M[u], inexact, q_ord + q * D, p_ord + jt * D,
+                               tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31));
             }
         }
     }
-    __syncthreads();
-#pragma unroll
-    for (int s = 0; s < kBPPW; s++) {
-        if (!act[s]) continue;
-        const bool any_tie = __any_sync(0xffffffffu, had_tie[s]);
-        const uint32_t *st = stw + s * G::WB;
-        uint32_t *out = rows32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
-        const uint32_t *tr = tie32 + (jt[s] >> 5) * (G::WB * 32) + (jt[s] & 31);
+    // consumer warps only (the producer has returned): named barrier 1
+    asm volatile("bar.sync 1, %0;" ::"r"(kBWarps * 32) : "memory");
+    for (int t = warp; t < nt; t += kBWarps) {
+        const int64_t jt = j0 + t;
+        const uint32_t *st = state + t * G::WB;
+        uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        const uint32_t *tr = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
         for (int w = lane; w < G::WB; w += 32) {
-            uint32_t v = st[w];
-            if (any_tie) v |= tr[w * 32];
+            const uint32_t v = st[w] | tr[w * 32];
             uint32_t row = ~v;
             if (w == 0) row &= ~1u;
             out[w * 32] = row;
             if (ext_rows32) {
                 uint32_t er = ~st[w];
                 if (w == 0) er &= ~1u;
-                ext_rows32[(jt[s] >> 5) * (G::WB * 32) + w * 32 + (jt[s] & 31)] = er;
+                ext_rows32[(jt >> 5) * (G::WB * 32) + w * 32 + (jt & 31)] = er;
             }
         }
     }
 }
 
-template <int D>
-void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+template <int D, bool TIES>
+void launch_a_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
-    const size_t smem = sizeof(uint32_t) * (4 * kAStages + kAStages * (size_t)kATQ * G::CW + (size_t)kAWarps * G::WB * 32);
-    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_a_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const size_t smem = sizeof(uint32_t) * (4 * kAStages + kAStages * (size_t)kATQ * G::CW +
+                                            (TIES ? 2 : 1) * (size_t)kAWarps * G::WB * 32);
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_a_kernel<D, TIES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int64_t ntq = ceil_div(c.m, kATQ);
     const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, kAWarps * 32);
-    k3_mdmc_a_kernel<D><<<blocks, (kAWarps + 1) * 32, smem, st>>>(
+    k3_mdmc_a_kernel<D, TIES><<<blocks, (kAWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(), ntq,
         j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
 
+// Tie-heavy inputs (every dimension discrete enough for injective codes) or small d keep the tie part of
+// B_{p notin S} in shared memory; otherwise ties are rare and go to a global row.
+template <int D>
+void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    const bool all_exact = c.exact_mask == ((1u << D) - 1u);
+    if (D <= 10 || all_exact) launch_a_t<D, true>(c, j_begin, j_end, rows32, ext_rows32, st);
+    else launch_a_t<D, false>(c, j_begin, j_end, rows32, ext_rows32, st);
+}
+
 template <int D>
 void launch_b(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
-    const size_t smem = sizeof(uint32_t) * ((size_t)kBTQ * G::CW + (size_t)kBWarps * kBPPW * G::WB);
+    constexpr int NT = GeoB<D>::NT;
+    const size_t smem = sizeof(uint32_t) * (4 * kBStages + kBStages * (size_t)kBTQ * G::CW + (size_t)NT * G::CW +
+                                            (size_t)NT * G::WB);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_b_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const int64_t ntq = ceil_div(c.m, kBTQ);
-    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, kBWarps * kBPPW);
-    k3_mdmc_b_kernel<D><<<blocks, kBWarps * 32, smem, st>>>(
+    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, NT);
+    k3_mdmc_b_kernel<D><<<blocks, (kBWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(), ntq,
         j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
     c.L.count++;
@@ -365,9 +407,7 @@ void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32
     const int d = c.d;
     const int cw = c.dp / 2;
     // q stream padding to whole tiles (both designs use tiles of at most 256)
-    const int64_t mpad = ceil_div(c.m, 256) * 256;
-    c.q_codes.ensure(sizeof(uint32_t) * mpad * cw);
-    c.q_ord.ensure(sizeof(uint32_t) * mpad * d);
+    const int64_t mpad = ceil_div(c.m, kQPad) * kQPad;  // capacity reserved by ext_build
     if (mpad > c.m) {
         pad_q_kernel<<<(unsigned)ceil_div(mpad - c.m, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(),
                                                                           c.m, mpad, cw, d);

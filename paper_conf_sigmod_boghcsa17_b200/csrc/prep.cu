@@ -232,8 +232,8 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.ext_ids.ensure(sizeof(int32_t) * mm);
     c.p_codes.ensure(sizeof(uint16_t) * (mm + 32) * c.dp);
     c.p_ord.ensure(sizeof(uint32_t) * mm * d);
-    c.q_codes.ensure(sizeof(uint16_t) * (mm + 1024) * c.dp);
-    c.q_ord.ensure(sizeof(uint32_t) * mm * d);
+    c.q_codes.ensure(sizeof(uint16_t) * (mm + kQPad) * c.dp);
+    c.q_ord.ensure(sizeof(uint32_t) * (mm + kQPad) * d);
     ext_build_id_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(),
                                                             c.codes_id.as<uint32_t>(), c.ord.as<uint32_t>(), n, d, cw,
                                                             c.ext_ids.as<int32_t>(), c.p_codes.as<uint32_t>(),

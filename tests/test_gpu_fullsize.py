@@ -1,0 +1,93 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times (pipeline.DeviceSkycube),
+on outputs the oracle can compute one by one (seeded samples of points), plus properties that hold at
+any size.  Needs a B200."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+SAMPLE = 48
+
+
+@pytest.fixture(scope="module")
+def engine():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_sigmod_boghcsa17_b200.pipeline import DeviceSkycube
+    eng = DeviceSkycube(0)
+    yield eng
+    eng.close()
+
+
+def _build(engine, x):
+    import torch
+    pts = torch.from_numpy(x).cuda()
+    out = engine.build(pts, lists=True, membership=True)
+    torch.cuda.synchronize()
+    return out
+
+
+def _rows_of(out, pids):
+    import torch
+    mem = out["membership"]
+    return mem[torch.as_tensor(pids, device=mem.device)].cpu().numpy().view(np.uint32)
+
+
+@pytest.mark.parametrize("name", ["C2", "C3C", "C3I", "C3A", "C5", "H", "C4"])
+def test_full_size_sampled_rows_and_lattice_properties(engine, name):
+    import torch
+    cfg = datagen.config(name)
+    x = cfg.data()
+    n, d = x.shape
+    out = _build(engine, x)
+    m = out["n_ext"]
+    rng = np.random.default_rng(1234)
+    ext_ids = out["ext_ids"].cpu().numpy()
+    assert np.all(np.diff(ext_ids) > 0) and len(ext_ids) == m
+    # half the sample from S+ (interesting rows), half uniform (mostly zero rows outside S+)
+    pids = np.unique(np.concatenate([rng.choice(ext_ids, SAMPLE // 2, replace=False),
+                                     rng.choice(n, SAMPLE // 2, replace=False)]))
+    want_rows, want_ext = oracle.rows_b(x, pids, with_ext=True)
+    got = _rows_of(out, pids)
+    bad = np.nonzero((got != want_rows).any(axis=1))[0]
+    assert bad.size == 0, f"{name}: rows of points {pids[bad][:5]} differ"
+    full = (1 << d) - 1
+    in_ext = ((want_ext[:, full >> 5] >> (full & 31)) & 1).astype(bool)
+    assert np.array_equal(np.isin(pids, ext_ids), in_ext), f"{name}: S+ membership differs on the sample"
+
+    # lattice properties at full size
+    off = out["offsets"].cpu().numpy()
+    nsub = 1 << d
+    assert off[0] == 0 and off[1] == 0 and np.all(np.diff(off) >= 0)
+    assert np.all(np.diff(off)[1:] >= 1), "I4: every subspace skyline is non-empty"
+    mem = out["membership"]
+    pop = sum(int(((mem >> b) & 1).sum(dtype=torch.int64).item()) for b in range(32))
+    assert pop == off[-1], "total ids == total membership bits"
+    ids = out["ids"]
+    deltas = sorted(set([1, 2, nsub - 1, nsub // 2 + 1] + rng.integers(1, nsub, 6).tolist()))
+    for delta in deltas:
+        lst = ids[off[delta]:off[delta + 1]].cpu().numpy()
+        assert np.all(np.diff(lst) > 0), f"ids ascending in delta {delta}"
+        word = mem[:, delta >> 5].cpu().numpy().view(np.uint32)
+        members = np.nonzero((word >> (delta & 31)) & 1)[0]
+        assert np.array_equal(lst, members), f"lattice of delta {delta} == transpose of rows"
+    # I1: rows outside S+ are zero
+    nz = torch.nonzero(mem.any(dim=1)).flatten().cpu().numpy()
+    assert np.all(np.isin(nz, ext_ids))
+
+
+def test_c2_full_oracle(engine):
+    x = datagen.config("C2").data()
+    out = _build(engine, x)
+    want = oracle.rows_b(x)
+    got = out["membership"].cpu().numpy().view(np.uint32)
+    assert np.array_equal(got, want)
+    offs, ids = oracle.lattice(want, x.shape[1])
+    assert np.array_equal(out["offsets"].cpu().numpy(), offs)
+    assert np.array_equal(out["ids"].cpu().numpy(), ids)
