@@ -49,6 +49,10 @@ def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
     return sms * 128 * sm_mhz * 1e6
 
 
+def workload(cfg) -> str:
+    return f"{cfg.name}: {cfg.dist} n={cfg.n} d={cfg.d} seed={cfg.seed} (datagen, Börzsönyi-style)"
+
+
 def env_rank():
     return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("LOCAL_RANK", "0"))
 
@@ -167,8 +171,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": full * 1e3, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {cfg.dist} n={cfg.n} d={cfg.d} seed={cfg.seed}", "n": cfg.n,
-                   "d": cfg.d, "n_ext_estimated": est_next},
+        "config": {"workload": workload(cfg), "n": cfg.n, "d": cfg.d, "n_ext_estimated": est_next},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": times[0][4], "kind": "oracle",
                          "sample": f"Oracle B (oracle/skycube_oracle.c) rows for {times[0][1]} uniformly sampled "
                                    f"points of {cfg.n} per step ({times[0][2]:.1f} s), extrapolated x n/sample; "
@@ -261,8 +264,7 @@ def run_ours(args):
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {cfg.dist} n={n} d={d} seed={cfg.seed} (datagen, Börzsönyi-style)",
-                   "n": n, "d": d, "n_ext": m, "pairs": pairs, "total_ids": total_ids,
+        "config": {"workload": workload(cfg), "n": n, "d": d, "n_ext": m, "pairs": pairs, "total_ids": total_ids,
                    "l2": "256 MB buffer written between timed steps",
                    "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
         "phases_ms": phase,
