@@ -103,15 +103,15 @@ skycube_status skycube_ctx_create(int32_t device, skycube_ctx **ctx);
 void skycube_ctx_destroy(skycube_ctx *ctx);
 
 /* Phase 1 (replicated on every rank): validate (K0: NaN -> ENAN, -0 -> +0, order-preserving keys),
- * sort by the exact key sum (Λ2), and compute per-dimension 15-bit monotone codes (K2).
+ * compute per-dimension 15-bit monotone codes (K2), and put the points in static-tree order (Morton order
+ * of the codes: the leaf order of the paper's global-pivot tree, L338) with 32-point chunk records.
  * d_points: [n*d] float32 row-major on the device. */
 skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, void *stream);
 
-/* Phase 2: extended-skyline prefilter (K1).  Sorted positions are cut into tiles of 256; this call
- * processes the tiles t with t % tile_step == tile_offset (interleaving balances ranks: later tiles
- * have longer candidate prefixes).  Writes d_ext_sorted[s] = 1 iff the point at key-sorted position s
- * is in S+(P), 0 otherwise, for the positions of those tiles only.
- * d_ext_sorted: [n] uint8 device buffer owned by the caller. */
+/* Phase 2: extended-skyline prefilter (K1).  The prepared (static-tree) positions are cut into blocks of
+ * 2048; this call processes the blocks b with b % tile_step == tile_offset (interleaving balances ranks).
+ * Writes d_ext_sorted[s] = 1 iff the point at prepared position s is in S+(P), 0 otherwise, for the
+ * positions of those blocks only.  d_ext_sorted: [n] uint8 device buffer owned by the caller. */
 skycube_status skycube_dev_prefilter(skycube_ctx *ctx, int64_t tile_offset, int64_t tile_step,
                                      uint8_t *d_ext_sorted, void *stream);
 

@@ -55,16 +55,19 @@ struct Ctx {
     DevBuf rbuf;        // u32 [kMaxD]
     DevBuf nanflag;     // u32 [1]
     DevBuf codes_id;    // u16 [n*dp]  id order
-    DevBuf codes_sorted;// u16 [n*dp]  key-sum order
-    DevBuf ord_sorted;  // u32 [n*d]   key-sum order
+    DevBuf codes_sorted;// u16 [npad*dp]  static-tree (Morton) order, padded to whole chunk tiles
+    DevBuf ord_sorted;  // u32 [n*d]      static-tree order
     // S+ (m points)
     DevBuf ext_id_flag, ext_idx, key_flag, key_idx;  // u32 [n]
     DevBuf ext_ids;     // i32 [m] ascending
     DevBuf p_codes;     // u16 [m*dp]  S+ in id order (MDMC tasks)
     DevBuf p_ord;       // u32 [m*d]
-    DevBuf q_codes;     // u16 [m*dp]  S+ in key-sum order (MDMC competitor stream)
+    DevBuf q_codes;     // u16 [mpad*dp]  S+ in static-tree order (MDMC competitor stream)
     DevBuf q_ord;       // u32 [m*d]
     DevBuf tie;         // u32 tiled rows: tie contributions to B_{p notin S}
+    DevBuf chunks_all;  // u32 [n/32][33][cw]  chunk records of all points (K1 competitors)
+    DevBuf chunks_ext;  // u32 [m/32][33][cw]  chunk records of S+ (K3 competitors)
+    int64_t nchunks_all = 0, nchunks_ext = 0;
     DevBuf lat_counts;  // u64 [2^d * nchunks]
     DevBuf scan64_tmp;
 };
@@ -83,5 +86,6 @@ void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *
 
 constexpr int kPrefilterTile = 256;  // sorted positions per K1 block
 constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
+constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole
 
 }  // namespace sky

@@ -2,110 +2,157 @@
 //
 //   p in S+(P)  <=>  no q in P strictly dominates p in the full space (Def. 1-2, delta = 2^d - 1).
 //
-// Λ2: key(x) = sum_i ord(x[i]) is exact in 64 bits and q strictly dominates p implies
-// key(q) < key(p).  Points are sorted by key (prep.cu), so a point at sorted position s only needs
-// the positions t < s as candidates; scanning them from the smallest key first finds the strong
-// dominators early, and a block stops as soon as every one of its points is dominated.
+// Competitors are all points in static-tree (Morton) order, in chunks of 32 with their lower corner
+// (per-dimension minimum code).  q < p in every dimension requires code(q) <= code(p), hence
+// corner < p in every dimension; a chunk whose corner fails that for a task cannot hold a dominator
+// of it (the mask test of Eq. 1, applied to a whole leaf range of the static tree).
 //
-// Each candidate is first rejected through the 15-bit codes: q < p in every dimension requires
-// code(q) <= code(p) in every dimension (Λ3), which is a SWAR test of 16-bit lanes with a guard bit
-// (two dimensions per 32-bit word; no branches).  Survivors get the exact test on the
-// order-preserving keys.
+// CTA: kTasks tasks (consecutive tree positions) with their codes in shared memory, 16 consumer warps
+// and one TMA producer warp streaming chunk tiles (16 chunk records per tile) through a 3-stage ring.
+// Each consumer warp takes one chunk per tile: its 32 competitors sit in registers (one per lane);
+//   box pass: lane l tests task tb+l against the chunk corner (SWAR strict compare, guard bits);
+//   a ballot gives the tasks that need pair tests; for each, all lanes test their competitor
+//   (codes strictly less in every dimension => dominated; equal codes in a non-injective dimension
+//   fall back to the exact keys).  A dominated task is marked in a shared bit set and skipped after.
 #include "ctx.cuh"
 #include "tile_stream.cuh"
 
 namespace sky {
 namespace {
 
-constexpr int kThreads = kPrefilterTile;  // one sorted position per thread
-constexpr int kTQ = 256;                  // candidates per shared-memory tile
-constexpr int kU = 4;                     // candidates per inner iteration
+constexpr int kWarps = 16;         // consumer warps = chunks per tile
+constexpr int kTasks = 2048;       // tasks per CTA
+constexpr int kStages = 3;
 
 template <int CW>
-__global__ void __launch_bounds__(kThreads) k1_prefilter_kernel(
-    const uint32_t *__restrict__ codes_sorted, const uint32_t *__restrict__ ord_sorted, int64_t n, int d,
-    int64_t tile_offset, int64_t tile_step, int64_t ntiles_mine, uint8_t *__restrict__ ext_sorted) {
+__global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
+    const uint32_t *__restrict__ codes_sorted, const uint32_t *__restrict__ chunks,
+    const uint32_t *__restrict__ ord_sorted, int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset,
+    int64_t blk_step, uint8_t *__restrict__ ext_sorted) {
+    constexpr int CWP = CW | 1;         // odd row stride: conflict-free per-lane task loads
+    constexpr int REC = 33 * CW;        // chunk record words
     extern __shared__ __align__(128) uint32_t smem[];
-    const TileStream2 ts{reinterpret_cast<uint64_t *>(smem), smem + 4, (uint32_t)(kTQ * CW)};
-    const int64_t tile = tile_offset + (ntiles_mine - 1 - (int64_t)blockIdx.x) * tile_step;  // heaviest first
-    const int64_t s = tile * kThreads + threadIdx.x;
-    const bool valid = s < n;
-    if (threadIdx.x == 0) ts.init();
-    uint32_t pH[CW];
-#pragma unroll
-    for (int k = 0; k < CW; k++) {
-        uint32_t w = valid ? codes_sorted[s * CW + k] : 0u;
-        // padding halves (dimensions >= d) must never reject: make p maximal there
-        if (2 * k >= d) w |= 0x00007fffu;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)(kWarps * REC)};
+    uint32_t *pH = smem + 4 * kStages + kStages * kWarps * REC;  // [kTasks][CWP]
+    uint32_t *domw = pH + kTasks * CWP;                           // [kTasks / 32] dominated bits
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t blk = blk_offset + (int64_t)blockIdx.x * blk_step;
+    const int64_t s0 = blk * kTasks;
+    const int nt = (int)min((int64_t)kTasks, n - s0);
+    const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
+
+    if (threadIdx.x == 0) ring.init(kWarps);
+    for (int i = threadIdx.x; i < kTasks * CW; i += blockDim.x) {
+        const int t = i / CW, k = i % CW;
+        uint32_t w = t < nt ? codes_sorted[(s0 + t) * CW + k] : 0u;
+        if (2 * k >= d) w |= 0x00007fffu;      // padding dimensions never reject
         if (2 * k + 1 >= d) w |= 0x7fff0000u;
-        pH[k] = w | kGuard;
+        pH[t * CWP + k] = w | kGuard;
     }
-    const int64_t s_hi = min(n, (tile + 1) * (int64_t)kThreads);
-    const int64_t nqt = ceil_div_dev(s_hi, kTQ);
+    for (int i = threadIdx.x; i < kTasks / 32; i += blockDim.x) {
+        uint32_t dead = 0;  // tasks past n count as dominated
+        for (int b = 0; b < 32; b++)
+            if (i * 32 + b >= nt) dead |= 1u << b;
+        domw[i] = dead;
+    }
     __syncthreads();
-    int64_t issued = 0;
-    if (threadIdx.x == 0) {
-        ts.issue(codes_sorted, 0);
-        if (nqt > 1) ts.issue(codes_sorted, 1);
+    if (warp == kWarps) {
+        if (lane == 0)
+            for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
+        return;
     }
-    issued = nqt > 1 ? 2 : 1;
-    bool dom = !valid;
-    int64_t qt = 0;
-    for (; qt < nqt; qt++) {
-        ts.wait(qt);
-        const uint32_t *qs = ts.stage(qt);
-        if (!dom) {
-#pragma unroll 1
-            for (int t = 0; t < kTQ; t += kU) {
-                uint32_t cand = 0;
+    // corner test: q < p needs code(q) < code(p) on injective dimensions but only code(q) <= code(p) on
+    // the others (a bin may hold several values), so subtract 1 only in the injective lanes
+    uint32_t csub[CW];
 #pragma unroll
-                for (int u = 0; u < kU; u++) {
-                    uint32_t acc = 0xffffffffu;
+    for (int k = 0; k < CW; k++)
+        csub[k] = (((inexact >> (2 * k)) & 1u) ? 0u : 1u) | (((inexact >> (2 * k + 1)) & 1u) ? 0u : 0x10000u);
+    const int ngroups = (nt + 31) >> 5;
+    for (int64_t tile = 0; tile < ntiles; tile++) {
+        ring.wait(tile);
+        const uint32_t *rec = ring.stage(tile) + warp * REC;
+        uint32_t q[CW], mn[CW];
 #pragma unroll
-                    for (int k = 0; k < CW; k++) acc &= pH[k] - qs[(t + u) * CW + k];  // guard <=> code(q) <= code(p)
-                    cand |= ((acc & kGuard) == kGuard) ? (1u << u) : 0u;
+        for (int k = 0; k < CW; k++) {
+            q[k] = rec[lane * CW + k];
+            mn[k] = rec[32 * CW + k];
+        }
+        __syncwarp();
+        if (lane == 0) ring.release(tile);
+        const int64_t c = tile * kWarps + warp;
+        if (c >= nchunks) continue;
+        const int64_t qpos = c * 32 + lane;
+        for (int g = 0; g < ngroups; g++) {
+            const int tt = g * 32 + lane;
+            const uint32_t dw = domw[g];
+            if (dw == 0xffffffffu) continue;
+            uint32_t acc = 0xffffffffu;
+#pragma unroll
+            for (int k = 0; k < CW; k++) acc &= pH[tt * CWP + k] - mn[k] - csub[k];  // corner below p
+            const bool cand = !((dw >> lane) & 1u) && (acc & kGuard) == kGuard;
+            uint32_t need = __ballot_sync(0xffffffffu, cand);
+            while (need) {
+                const int b = __ffs(need) - 1;
+                need &= need - 1;
+                const int ts = g * 32 + b;
+                const uint32_t *ph = pH + ts * CWP;
+                uint32_t lt = 0xffffffffu, le = 0xffffffffu;
+#pragma unroll
+                for (int k = 0; k < CW; k++) {
+                    const uint32_t x = ph[k] - q[k];
+                    le &= x;
+                    lt &= x - 0x00010001u;
                 }
-                if (cand == 0) continue;
+                bool dom = (lt & kGuard) == kGuard;  // codes strictly smaller everywhere
+                if (!dom && (le & kGuard) == kGuard && inexact) {
+                    // equal codes somewhere: only non-injective dimensions may still be strictly less
+                    dom = true;
+                    const int64_t ps = s0 + ts;
 #pragma unroll
-                for (int u = 0; u < kU; u++) {
-                    const int64_t q = qt * kTQ + t + u;
-                    if (((cand >> u) & 1u) && q < s && !dom) {
-                        bool strict = true;
-                        for (int i = 0; i < d && strict; i++) strict = ord_sorted[q * d + i] < ord_sorted[s * d + i];
-                        dom = strict;
+                    for (int k = 0; k < CW; k++) {
+#pragma unroll
+                        for (int h = 0; h < 2; h++) {
+                            const int i = 2 * k + h;
+                            if (i >= d) continue;
+                            const uint32_t qc = (q[k] >> (16 * h)) & 0xffffu, pc = (ph[k] >> (16 * h)) & 0x7fffu;
+                            if (qc != pc) continue;
+                            if (!((inexact >> i) & 1u) || !(ord_sorted[qpos * d + i] < ord_sorted[ps * d + i]))
+                                dom = false;
+                        }
                     }
                 }
-                if (dom) break;
+                if (__any_sync(0xffffffffu, dom) && lane == 0) atomicOr(&domw[ts >> 5], 1u << (ts & 31));
             }
         }
-        const int all = __syncthreads_and(dom);
-        if (all) break;
-        if (threadIdx.x == 0 && qt + 2 < nqt) ts.issue(codes_sorted, qt + 2);
-        issued = min(nqt, qt + 3);
     }
-    // drain bulk copies still in flight before the CTA's shared memory is released
-    if (threadIdx.x == 0)
-        for (int64_t t = qt + 1; t < issued; t++) ts.wait(t);
-    if (valid) ext_sorted[s] = dom ? 0 : 1;
+    asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32) : "memory");
+    for (int t = threadIdx.x; t < nt; t += kWarps * 32) ext_sorted[s0 + t] = ((domw[t >> 5] >> (t & 31)) & 1u) ? 0 : 1;
 }
 
 template <int CW>
-void launch(Ctx &c, int64_t tile_offset, int64_t tile_step, int64_t ntiles_mine, uint8_t *ext, cudaStream_t st) {
-    const size_t smem = sizeof(uint32_t) * (4 + 2 * (size_t)kTQ * CW);
-    k1_prefilter_kernel<CW><<<(unsigned)ntiles_mine, kThreads, smem, st>>>(
-        c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, tile_offset, tile_step, ntiles_mine, ext);
+void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uint8_t *ext, cudaStream_t st) {
+    constexpr int CWP = CW | 1;
+    const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * kWarps * 33 * CW + (size_t)kTasks * CWP +
+                                            kTasks / 32);
+    SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
+    k1_prefilter_kernel<CW><<<(unsigned)nblk_mine, (kWarps + 1) * 32, smem, st>>>(
+        c.codes_sorted.as<uint32_t>(), c.chunks_all.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, inexact,
+        c.nchunks_all, blk_offset, blk_step, ext);
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
 
 }  // namespace
 
+// Blocks of kTasks consecutive tree positions; block b is processed iff b % tile_step == tile_offset.
 void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ext_sorted, cudaStream_t st) {
     if (!c.prepared) throw Error{1, "skycube_dev_prefilter before skycube_dev_prepare"};
-    if (tile_step < 1 || tile_offset < 0) throw Error{1, "bad prefilter tile range"};
-    const int64_t ntiles = ceil_div(c.n, kThreads);
-    if (tile_offset >= ntiles) return;
-    const int64_t mine = (ntiles - 1 - tile_offset) / tile_step + 1;
+    if (tile_step < 1 || tile_offset < 0) throw Error{1, "bad prefilter block range"};
+    const int64_t nblk = ceil_div(c.n, kTasks);
+    if (tile_offset >= nblk) return;
+    const int64_t mine = (nblk - 1 - tile_offset) / tile_step + 1;
     switch (c.dp / 2) {
         case 2: launch<2>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
         case 4: launch<4>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
@@ -114,5 +161,7 @@ void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ex
         default: throw Error{1, "unsupported dimensionality"};
     }
 }
+
+int64_t prefilter_block_size() { return kTasks; }
 
 }  // namespace sky

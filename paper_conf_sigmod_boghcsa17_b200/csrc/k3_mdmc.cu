@@ -25,6 +25,8 @@
 //   design B (d > 12): a CTA holds the states of NT tasks (192 KB in total, 8 KB per task at d = 16);
 //     each lane holds one competitor in registers and runs it against all NT tasks (task codes are
 //     broadcasts); misses expand with shared-memory atomics.
+#include <cstdlib>
+
 #include "ctx.cuh"
 #include "tile_stream.cuh"
 
@@ -350,6 +352,198 @@ __global__ void __launch_bounds__((kBWarps + 1) * 32, 1) k3_mdmc_b_kernel(
     }
 }
 
+// ==================================================================================== design C
+// Static-tree chunk pruning (any d).  Competitors are S+ in static-tree (Morton) order, in chunks of 32
+// with their lower corner.  For a task p and a chunk, Mbox = B_{corner<=p} is a superset of M(q,p) for
+// every q of the chunk, so bit Mbox set in B_{p notin S+} proves the whole chunk adds nothing (Λ4 on a
+// leaf range: the paper's filter on path labels, L320-328, with the tree's global pivots).  A CTA holds
+// NT tasks; each consumer warp takes one chunk per tile (one competitor per lane, in registers):
+//   box pass   lane l tests task g*32+l against the chunk corner; a ballot gives the tasks to refine;
+//   pair pass  for each such task (4 at a time) every lane tests its competitor (task codes are a
+//              shared-memory broadcast) and probes the task's state; misses run Alg. 3 lines 10-12 with
+//              shared-memory atomics (several warps may update one task).
+constexpr int kCWarps = 16;
+constexpr int kCStages = 3;
+constexpr int kCStateBytes = 144 * 1024;
+constexpr int kCU = 4;
+
+template <int D, bool TIES>
+struct GeoC {
+    static constexpr int PER = (TIES ? 2 : 1) * Geo<D>::WB;       // state words per task
+    static constexpr int NT0 = kCStateBytes / (PER * 4);
+    static constexpr int NT = NT0 < 1024 ? NT0 : 1024;            // tasks per CTA
+};
+
+template <int D, bool TIES>
+__device__ __forceinline__ void mdmc_miss_c(uint32_t *st, const uint32_t *ph, const uint32_t *q, uint32_t M,
+                                            uint32_t inexact, const uint32_t *__restrict__ qo,
+                                            const uint32_t *__restrict__ po, uint32_t *tr, int tstride) {
+    using G = Geo<D>;
+    uint32_t lt[G::CW];
+#pragma unroll
+    for (int k = 0; k < G::CW; k++) lt[k] = ph[k] - q[k] - 0x00010001u;
+    uint32_t S = gather_mask<G::NG>(lt);
+    uint32_t L = M;
+    const uint32_t U = M & ~S & inexact;
+    if (U) refine_exact(U, qo, po, L, S);
+    if (S == 0) return;
+    if (L != M && ((st[L >> 5] >> (L & 31)) & 1u)) return;
+    if (!((st[S >> 5] >> (S & 31)) & 1u)) {
+        const uint32_t sh = S >> 5, bits = sub5(S & 31u);
+        uint32_t w = 0;
+        do {
+            atomicOr(&st[w], bits);
+            w = (w - sh) & sh;
+        } while (w);
+    }
+    if (L == S) return;
+    const uint32_t E = L & ~S;
+    const uint32_t lh = L >> 5, eh = E >> 5, lb = sub5(L & 31u), eb = sub5(E & 31u);
+    uint32_t w = 0;
+    do {
+        atomicOr(&tr[w * tstride], (w & ~eh) ? lb : (lb & ~eb));
+        w = (w - lh) & lh;
+    } while (w);
+}
+
+template <int D, bool TIES>
+__global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
+    const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
+    const uint32_t *__restrict__ q_ord, int64_t nchunks, int64_t j_begin, int64_t j_end, uint32_t inexact,
+    uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
+    using G = Geo<D>;
+    using C = GeoC<D, TIES>;
+    constexpr int CWP = G::CW | 1;
+    constexpr int REC = 33 * G::CW;
+    extern __shared__ __align__(128) uint32_t smem[];
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    const TileRing<kCStages> ring{bars, bars + kCStages, smem + 4 * kCStages, (uint32_t)(kCWarps * REC)};
+    uint32_t *pH = smem + 4 * kCStages + kCStages * kCWarps * REC;  // [NT][CWP]
+    uint32_t *state = pH + C::NT * CWP;                              // [NT][PER]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t j0 = j_begin + (int64_t)blockIdx.x * C::NT;
+    const int nt = (int)min((int64_t)C::NT, j_end - j0);
+    const int64_t ntiles = ceil_div_dev(nchunks, kCWarps);
+
+    if (threadIdx.x == 0) ring.init(kCWarps);
+    for (int i = threadIdx.x; i < C::NT * G::CW; i += blockDim.x) {
+        const int t = i / G::CW, k = i % G::CW;
+        uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
+        if (2 * k >= D) w &= 0xffff0000u;  // padding dimensions: p = 0 never passes q <= p (q pad = 1)
+        if (2 * k + 1 >= D) w &= 0x0000ffffu;
+        pH[t * CWP + k] = w | kGuard;
+    }
+    for (int i = threadIdx.x; i < C::NT * C::PER; i += blockDim.x) state[i] = (i % C::PER) == 0 ? 1u : 0u;
+    __syncthreads();
+    if (warp == kCWarps) {
+        if (lane == 0)
+            for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
+        return;
+    }
+    const int ngroups = (nt + 31) >> 5;
+    for (int64_t tile = 0; tile < ntiles; tile++) {
+        ring.wait(tile);
+        const uint32_t *rec = ring.stage(tile) + warp * REC;
+        uint32_t q[G::CW], mn[G::CW];
+#pragma unroll
+        for (int k = 0; k < G::CW; k++) {
+            q[k] = rec[lane * G::CW + k];
+            mn[k] = rec[32 * G::CW + k];
+        }
+        __syncwarp();
+        if (lane == 0) ring.release(tile);
+        const int64_t c = tile * kCWarps + warp;
+        if (c >= nchunks) continue;
+        const int64_t qpos = c * 32 + lane;
+        for (int g = 0; g < ngroups; g++) {
+            const int tt = min(g * 32 + lane, nt - 1);
+            uint32_t le[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
+            const uint32_t Mb = gather_mask<G::NG>(le);
+            const uint32_t wb = state[tt * C::PER + (Mb >> 5)];
+            const bool need = g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
+            uint32_t todo = __ballot_sync(0xffffffffu, need);
+            while (todo) {
+                int ts[kCU];
+                int cnt = 0;
+#pragma unroll
+                for (int u = 0; u < kCU; u++) {
+                    ts[u] = g * 32 + (todo ? __ffs(todo) - 1 : 0);
+                    if (todo) {
+                        todo &= todo - 1;
+                        cnt++;
+                    }
+                }
+                uint32_t M[kCU], wd[kCU];
+#pragma unroll
+                for (int u = 0; u < kCU; u++) {
+                    const uint32_t *ph = pH + ts[u] * CWP;
+                    uint32_t x[G::CW];
+#pragma unroll
+                    for (int k = 0; k < G::CW; k++) x[k] = ph[k] - q[k];
+                    M[u] = gather_mask<G::NG>(x);
+                    wd[u] = state[ts[u] * C::PER + (M[u] >> 5)];
+                }
+                uint32_t hit = 0xffffffffu;
+#pragma unroll
+                for (int u = 0; u < kCU; u++) hit &= __funnelshift_r(wd[u], wd[u], M[u]);
+                if (hit & 1u) continue;
+#pragma unroll
+                for (int u = 0; u < kCU; u++) {
+                    if (u >= cnt) break;
+                    uint32_t *st = state + ts[u] * C::PER;
+                    if ((st[M[u] >> 5] >> (M[u] & 31)) & 1u) continue;
+                    const int64_t jt = j0 + ts[u];
+                    uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+                    mdmc_miss_c<D, TIES>(st, pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D,
+                                         tr, TIES ? 1 : 32);
+                }
+            }
+        }
+    }
+    asm volatile("bar.sync 1, %0;" ::"r"(kCWarps * 32) : "memory");
+    for (int t = warp; t < nt; t += kCWarps) {
+        const int64_t jt = j0 + t;
+        const uint32_t *st = state + t * C::PER;
+        uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        const uint32_t *trg = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        for (int w = lane; w < G::WB; w += 32) {
+            const uint32_t v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+            uint32_t row = ~v & G::kRowMask;
+            if (w == 0) row &= ~1u;
+            out[w * 32] = row;
+            if (ext_rows32) {
+                uint32_t er = ~st[w] & G::kRowMask;
+                if (w == 0) er &= ~1u;
+                ext_rows32[(jt >> 5) * (G::WB * 32) + w * 32 + (jt & 31)] = er;
+            }
+        }
+    }
+}
+
+template <int D, bool TIES>
+void launch_c_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    using G = Geo<D>;
+    using C = GeoC<D, TIES>;
+    const size_t smem = sizeof(uint32_t) * (4 * kCStages + (size_t)kCStages * kCWarps * 33 * G::CW +
+                                            (size_t)C::NT * (G::CW | 1) + (size_t)C::NT * C::PER);
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_c_kernel<D, TIES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, C::NT);
+    k3_mdmc_c_kernel<D, TIES><<<blocks, (kCWarps + 1) * 32, smem, st>>>(
+        c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
+        c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
+template <int D>
+void launch_c(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    const bool all_exact = c.exact_mask == ((1u << D) - 1u);
+    if (D <= 10 || all_exact) launch_c_t<D, true>(c, j_begin, j_end, rows32, ext_rows32, st);
+    else launch_c_t<D, false>(c, j_begin, j_end, rows32, ext_rows32, st);
+}
+
 template <int D, bool TIES>
 void launch_a_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
@@ -418,6 +612,18 @@ void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32
     const size_t grp_words = (size_t)c.W * 32;
     c.tie.ensure(sizeof(uint32_t) * grp_words * (size_t)ceil_div(c.m, 32));
     SKY_CUDA(cudaMemsetAsync(c.tie.as<uint32_t>() + g0 * grp_words, 0, sizeof(uint32_t) * grp_words * (g1 - g0), st));
+    const char *sel = getenv("SKYCUBE_K3");
+    const char design = sel && *sel ? sel[0] : 'c';
+    if (design == 'c') {
+        switch (d) {
+#define SKY_C(DD) case DD: launch_c<DD>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+            SKY_C(1) SKY_C(2) SKY_C(3) SKY_C(4) SKY_C(5) SKY_C(6) SKY_C(7) SKY_C(8)
+            SKY_C(9) SKY_C(10) SKY_C(11) SKY_C(12) SKY_C(13) SKY_C(14) SKY_C(15) SKY_C(16)
+#undef SKY_C
+            default: throw Error{1, "d must be in [1, 16]"};
+        }
+        return;
+    }
     switch (d) {
         case 1: launch_a<1>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
         case 2: launch_a<2>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;

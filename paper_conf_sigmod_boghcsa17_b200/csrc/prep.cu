@@ -8,6 +8,12 @@
 // per-dimension bins — but with 2^15 bins per dimension (dense ranks, made coarser only when a
 // dimension has more than 2^15 distinct values), so that the bin comparison is exact for any
 // dimension with <= 2^15 distinct values and almost always decisive otherwise.
+//
+// The leaves of the paper's static tree, in order, are reproduced by sorting the points on the Morton
+// (bit-interleaved) key of their codes, top bits first: bit 1 of every dimension is the median split,
+// bit 2 the quartile split, ... (L338 "median, then quartile, then octile").  Consecutive runs of 32
+// points in that order are "chunks" whose per-dimension minimum codes bound every member; K1 and K3
+// test a whole chunk against a task with one mask test (Eq. 1's idea, L1312) before any pair.
 #include "ctx.cuh"
 
 namespace sky {
@@ -22,25 +28,59 @@ __device__ __forceinline__ uint32_t ord_key(float x) {
 
 // K0: one thread per point.
 __global__ void k0_canon_kernel(const float *__restrict__ pts, int64_t n, int d, uint32_t *__restrict__ ord,
-                                uint64_t *__restrict__ keysum, uint32_t *__restrict__ perm,
                                 uint64_t *__restrict__ comp_keys, uint32_t *__restrict__ comp_vals,
                                 uint32_t *__restrict__ nanflag) {
     const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
-    uint64_t s = 0;
     bool nan = false;
     for (int i = 0; i < d; i++) {
         const float x = pts[p * d + i];
         nan |= (x != x);
         const uint32_t o = ord_key(x);
         ord[p * d + i] = o;
-        s += o;                                      // exact: d * 2^32 < 2^37 (Λ2)
         comp_keys[(int64_t)i * n + p] = ((uint64_t)i << 32) | o;
         comp_vals[(int64_t)i * n + p] = (uint32_t)p;
     }
-    keysum[p] = s;
-    perm[p] = (uint32_t)p;
     if (nan) atomicOr(nanflag, 1u);
+}
+
+// Morton key of the codes, rescaled to the full 15-bit range (exact dimensions have codes < R):
+// bits_per_dim most significant bits of every dimension, interleaved, most significant level first.
+__global__ void morton_kernel(const uint16_t *__restrict__ codes, const uint32_t *__restrict__ R, int64_t n, int d,
+                              int dp, int bits_per_dim, uint64_t *__restrict__ keys, uint32_t *__restrict__ perm) {
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= n) return;
+    uint32_t sc[kMaxD];
+    for (int i = 0; i < d; i++) {
+        const uint32_t c = codes[p * dp + i], r = R[i];
+        sc[i] = r <= kCodeLevels ? (uint32_t)(((uint64_t)c * kCodeLevels) / r) : c;
+    }
+    uint64_t key = 0;
+    for (int b = 0; b < bits_per_dim; b++)
+        for (int i = 0; i < d; i++) key = (key << 1) | ((sc[i] >> (14 - b)) & 1u);
+    keys[p] = key;
+    perm[p] = (uint32_t)p;
+}
+
+// Chunk records: 32 consecutive points' code words, then the per-dimension minimum code words
+// (the chunk's lower corner).  One warp per chunk.
+__global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw,
+                                    uint32_t *__restrict__ chunks) {
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (c >= nchunks) return;
+    uint32_t *rec = chunks + c * (int64_t)(33 * cw);
+    for (int k = 0; k < cw; k++) {
+        const uint32_t w = codes[(c * 32 + lane) * cw + k];
+        rec[lane * cw + k] = w;
+        uint32_t lo = w & 0xffffu, hi = w >> 16;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+            hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+        }
+        if (lane == 0) rec[32 * cw + k] = lo | (hi << 16);
+    }
 }
 
 // flags[t] = 1 iff t starts a run of equal (dim, key) in the per-dimension sorted order.
@@ -86,8 +126,8 @@ __global__ void gather_sorted_kernel(const uint32_t *__restrict__ perm, const ui
                                      const uint32_t *__restrict__ ord, int64_t n, int d, int cw,
                                      uint32_t *__restrict__ codes_sorted, uint32_t *__restrict__ ord_sorted) {
     const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (s >= n) {  // padding up to whole K1 tiles: codes that never pass the q <= p test
-        if (s < ((n + 255) / 256) * 256)
+    if (s >= n) {  // padding up to whole chunks: codes that are never better than a task
+        if (s < ((n + 31) / 32) * 32)
             for (int k = 0; k < cw; k++) codes_sorted[s * cw + k] = 0x7fff7fffu;
         return;
     }
@@ -130,6 +170,26 @@ __global__ void ext_build_key_kernel(const uint32_t *__restrict__ key_flag, cons
 
 inline unsigned blocks_for(int64_t n, int t) { return (unsigned)ceil_div(n > 0 ? n : 1, t); }
 
+__global__ void fill_kernel(uint32_t *a, int64_t from, int64_t to, uint32_t v) {
+    const int64_t i = from + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < to) a[i] = v;
+}
+
+// "never better" padding: codes 0x7fff in every lane, keys above every finite value
+void pad_codes(uint32_t *codes, int64_t from, int64_t to, int cw, cudaStream_t st, Launches &L) {
+    if (to <= from) return;
+    fill_kernel<<<blocks_for((to - from) * cw, 256), 256, 0, st>>>(codes, from * cw, to * cw, 0x7fff7fffu);
+    L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
+void pad_ord(uint32_t *ord, int64_t from, int64_t to, int d, cudaStream_t st, Launches &L) {
+    if (to <= from) return;
+    fill_kernel<<<blocks_for((to - from) * d, 256), 256, 0, st>>>(ord, from * d, to * d, 0xffffffffu);
+    L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
 }  // namespace
 
 void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) {
@@ -142,6 +202,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.m = 0;
     const int64_t nd = n * d;
     const int cw = c.dp / 2;  // 32-bit code words per point
+    const int64_t npad = ceil_div(n, 32) * 32 + kChunkTilePad;  // whole chunks + whole chunk tiles
     c.ord.ensure(sizeof(uint32_t) * nd);
     c.keysum.ensure(sizeof(uint64_t) * n);
     c.perm.ensure(sizeof(uint32_t) * n);
@@ -156,12 +217,12 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
     c.nanflag.ensure(sizeof(uint32_t));
     c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
-    c.codes_sorted.ensure(sizeof(uint16_t) * (n + 256) * c.dp);
+    c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
     c.ord_sorted.ensure(sizeof(uint32_t) * nd);
+    c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * 33 * cw);
 
     SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
-    k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, c.ord.as<uint32_t>(), c.keysum.as<uint64_t>(),
-                                                        c.perm.as<uint32_t>(), c.comp_keys.as<uint64_t>(),
+    k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, c.ord.as<uint32_t>(), c.comp_keys.as<uint64_t>(),
                                                         c.comp_vals.as<uint32_t>(), c.nanflag.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
@@ -170,9 +231,6 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     SKY_CUDA(cudaStreamSynchronize(st));
     if (nan) throw Error{2, "NaN in input points"};
 
-    // Λ2 order: sum of order-preserving keys (< 2^36 for d <= 16), stable by id.
-    radix_sort_u64(c.keysum.as<uint64_t>(), c.perm.as<uint32_t>(), n, 36, c.keys_alt.as<uint64_t>(),
-                   c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
     // K2: per-dimension sort of (dim, key) -> dense ranks -> codes.
     radix_sort_u64(c.comp_keys.as<uint64_t>(), c.comp_vals.as<uint32_t>(), nd, 36, c.keys_alt.as<uint64_t>(),
                    c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
@@ -194,11 +252,26 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
         SKY_LAUNCH_CHECK();
     }
     SKY_CUDA(cudaMemcpyAsync(c.R, c.rbuf.p, sizeof(uint32_t) * d, cudaMemcpyDeviceToHost, st));
-    gather_sorted_kernel<<<blocks_for(n, 256) + 1, 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
-                                                             c.ord.as<uint32_t>(), n, d, cw,
-                                                             c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>());
+    // static-tree leaf order: Morton key of the codes (top bits first), then chunks of 32
+    const int bits_per_dim = std::min(15, 64 / d);
+    morton_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.codes_id.as<uint16_t>(), c.rbuf.as<uint32_t>(), n, d, c.dp,
+                                                      bits_per_dim, c.keysum.as<uint64_t>(), c.perm.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
+    radix_sort_u64(c.keysum.as<uint64_t>(), c.perm.as<uint32_t>(), n, bits_per_dim * d, c.keys_alt.as<uint64_t>(),
+                   c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
+    gather_sorted_kernel<<<blocks_for(npad, 256), 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
+                                                               c.ord.as<uint32_t>(), n, d, cw,
+                                                               c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    const int64_t nch = ceil_div(n, 32);
+    pad_codes(c.codes_sorted.as<uint32_t>(), nch * 32, npad, cw, st, c.L);
+    build_chunks_kernel<<<blocks_for((npad / 32) * 32, 256), 256, 0, st>>>(c.codes_sorted.as<uint32_t>(), npad / 32, cw,
+                                                                          c.chunks_all.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    c.nchunks_all = nch;
     SKY_CUDA(cudaStreamSynchronize(st));
     c.exact_mask = 0;
     for (int i = 0; i < d; i++)
@@ -229,22 +302,32 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     const int64_t m = (int64_t)last[0] + last[1];
     c.m = m;
     const int64_t mm = m > 0 ? m : 1;
+    const int64_t mpad = ceil_div(mm, kQPad) * kQPad;  // whole tiles of every K3 design
     c.ext_ids.ensure(sizeof(int32_t) * mm);
     c.p_codes.ensure(sizeof(uint16_t) * (mm + 32) * c.dp);
     c.p_ord.ensure(sizeof(uint32_t) * mm * d);
-    c.q_codes.ensure(sizeof(uint16_t) * (mm + kQPad) * c.dp);
-    c.q_ord.ensure(sizeof(uint32_t) * (mm + kQPad) * d);
+    c.q_codes.ensure(sizeof(uint16_t) * mpad * c.dp);
+    c.q_ord.ensure(sizeof(uint32_t) * mpad * d);
+    c.chunks_ext.ensure(sizeof(uint32_t) * (mpad / 32) * 33 * cw);
     ext_build_id_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(),
                                                             c.codes_id.as<uint32_t>(), c.ord.as<uint32_t>(), n, d, cw,
                                                             c.ext_ids.as<int32_t>(), c.p_codes.as<uint32_t>(),
                                                             c.p_ord.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
+    // competitor stream: S+ in static-tree (Morton) order, padded with never-better points
     ext_build_key_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.key_flag.as<uint32_t>(), c.key_idx.as<uint32_t>(),
                                                              c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>(),
                                                              n, d, cw, c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
+    pad_codes(c.q_codes.as<uint32_t>(), m, mpad, cw, st, c.L);
+    pad_ord(c.q_ord.as<uint32_t>(), m, mpad, d, st, c.L);
+    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw,
+                                                              c.chunks_ext.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    c.nchunks_ext = ceil_div(m, 32);
     c.ext_ready = true;
 }
 

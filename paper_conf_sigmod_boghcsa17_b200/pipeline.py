@@ -4,8 +4,8 @@ Sharding (the paper's device-level data parallelism of MDMC, L
 task is independent, there is no need for synchronisation"):
 
   1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic)
-  2. K1 prefilter                                 key-sorted tiles of 256 positions, tile t on rank
-                                                  t % world (interleaved: later tiles scan longer prefixes)
+  2. K1 prefilter                                 blocks of 2048 prepared (static-tree order) positions,
+                                                  block b on rank b % world
   3. exchange S+ flags                            all_reduce(MAX) of a uint8 flag vector (NCCL over NVLink)
   4. install S+ (replicated)
   5. K3 MDMC                                      contiguous ranges of 32-point groups of S+ (per-task cost is
@@ -26,13 +26,13 @@ import torch.distributed as dist
 
 from . import Context, words_per_row
 
-PREFILTER_TILE = 256
+PREFILTER_BLOCK = 2048  # prepared positions per K1 CTA (k1_prefilter.cu kTasks)
 GROUP = 32
 
 
 # ------------------------------------------------------------------ pure sharding arithmetic
 def prefilter_assignment(rank: int, world: int):
-    """(tile_offset, tile_step) of the K1 tiles a rank processes."""
+    """(block_offset, block_step) of the K1 blocks a rank processes."""
     return rank, world
 
 

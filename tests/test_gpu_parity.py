@@ -101,9 +101,22 @@ def test_inexact_codes_refinement():
     base = rng.integers(0, 1 << 20, size=(n, d)).astype(np.float32)
     x = np.ascontiguousarray(base)
     r = gpu(x)
+    assert np.array_equal(r["ext_ids"], np.nonzero(oracle.ext_full(x))[0])
     pids = rng.choice(n, 300, replace=False)
     want = oracle.rows_b(x, pids)
     assert np.array_equal(r["rows"][pids], want)
+
+
+@pytest.mark.parametrize("dist,d", [("A", 6), ("I", 5), ("C", 7)])
+def test_inexact_codes_continuous(dist, d):
+    # n > 2^15 distinct float values per dimension: non-injective codes on every dimension
+    n = 50000
+    x = datagen.generate(dist, n, d, 77)
+    r = gpu(x)
+    assert np.array_equal(r["ext_ids"], np.nonzero(oracle.ext_full(x))[0])
+    rng = np.random.default_rng(3)
+    pids = np.concatenate([rng.choice(r["ext_ids"], 150), rng.choice(n, 50)])
+    assert np.array_equal(r["rows"][pids], oracle.rows_b(x, pids))
 
 
 def test_edge_cases():
