@@ -35,10 +35,10 @@ UNIT = "dominance tests/s"
 L2_FLUSH_BYTES = 256 << 20
 
 
-def algorithmic_ops_per_pair(d: int) -> int:
-    """per ordered S+ pair, the two relation masks of Def. 1 (one compare per
-    dimension each: 2d) plus the probe of B_{p notin S+} (one load + one bit test: 2)."""
-    return 2 * d + 2
+def algorithmic_ops_per_test(d: int) -> int:
+    """DESIGN.md §5 Roofline: one test of K3 (a chunk-corner test or a pair test) forms the d-bit mask
+    B_{code<=code} (one compare per dimension: d) and probes B_{p notin S+} (one load + one bit test: 2)."""
+    return d + 2
 
 
 def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
@@ -217,6 +217,7 @@ def run_ours(args):
     total_ids = out["total_ids"]
     ev = [{k: torch.cuda.Event(enable_timing=True) for k in names} for _ in range(args.steps)]
     launches0 = eng.launches
+    cnt0 = eng.ctx.counters()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -232,6 +233,8 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
     launches = eng.launches - launches0
+    cnt1 = eng.ctx.counters()
+    work = {k: (cnt1[k] - cnt0[k]) / args.steps for k in cnt1}
     step_ms = [ev[s]["t0"].elapsed_time(ev[s]["t4"]) for s in range(args.steps)]
     phase = {k: statistics.mean(ev[s][a].elapsed_time(ev[s][b]) for s in range(args.steps))
              for k, a, b in [("prepare", "t0", "t1"), ("prefilter", "t1", "t2"), ("mdmc", "t2", "t3"),
@@ -254,10 +257,11 @@ def run_ours(args):
         return
     clocks = clk.summary()
     sm_mhz = clocks["sm_mhz"] or 1965.0
-    # roofline of the dominant kernel (K3 MDMC), duration from CUDA events on its stream
+    # roofline of the dominant kernel (K3 MDMC), duration from CUDA events on its stream; its work is
+    # the tests it must run after static-tree pruning (device counters), not the n_ext^2 pairs it resolves
     mdmc_ms = phase["mdmc"]
-    my_pairs = pairs if world == 1 else pairs / world
-    ops = my_pairs * algorithmic_ops_per_pair(d)
+    tests = work["k3_box"] + work["k3_pair"]
+    ops = tests * algorithmic_ops_per_test(d)
     achieved = ops / (mdmc_ms / 1e3) / 1e12
     peak = alu_peak_ops(sm_mhz) / 1e12
     line = {
@@ -268,10 +272,11 @@ def run_ours(args):
                    "l2": "256 MB buffer written between timed steps",
                    "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
         "phases_ms": phase,
+        "work_per_step": {**work, "pairs_resolved_by_chunk_tests": 32 * work["k3_box"] - work["k3_pair"]},
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
                      "frac": achieved / peak, "traffic": None,
-                     "kernel": "k3_mdmc", "ops_per_pair": algorithmic_ops_per_pair(d),
+                     "kernel": "k3_mdmc", "ops_per_test": algorithmic_ops_per_test(d), "tests": tests,
                      "peak_basis": f"148 SM x 128 integer lanes/clk (ALU+FMA pipes, 1 warp-inst/SMSP/clk) x {sm_mhz:.0f} MHz "
                                    f"(median SM clock under load)"},
         "clocks": clocks,

@@ -138,6 +138,12 @@ skycube_status skycube_dev_compact(skycube_ctx *ctx, const uint32_t *d_rows32, u
 /* Number of kernels launched by this context since creation (for the benchmark's gpu_launches). */
 int64_t skycube_ctx_launches(const skycube_ctx *ctx);
 
+/* Work counters accumulated by the context since creation (device-side, read with a sync):
+ * out8[0] K1 chunk-corner tests, [1] K1 pair tests, [2] K3 chunk-corner tests, [3] K3 pair tests,
+ * [4] K3 misses (pairs that reached Alg. 3 lines 10-12), [5..7] reserved (0).  Used by the benchmark's
+ * roofline (algorithmic work actually required after pruning). */
+skycube_status skycube_ctx_counters(const skycube_ctx *ctx, int64_t *out8);
+
 /* Problem facts after prepare / set_ext: n_ext (0 before set_ext), words per row, and the bit mask of
  * dimensions whose 15-bit codes are injective (exact). Any pointer may be NULL. */
 skycube_status skycube_ctx_info(const skycube_ctx *ctx, int64_t *n_ext, uint32_t *words_per_row,

@@ -14,7 +14,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libskycube.so")
+LIB_PATH = os.environ.get("SKYCUBE_LIB") or os.path.join(_PKG, "libskycube.so")
 
 OK, EINVAL, ENAN, ENOMEM, ECUDA, ENCCL, ENODEV = range(7)
 NO_LISTS = 0x1
@@ -24,7 +24,7 @@ EXPORTED = (
     "skycube_build", "skycube_build_ex", "skycube_free", "skycube_strerror", "skycube_last_error",
     "skycube_ctx_create", "skycube_ctx_destroy", "skycube_dev_prepare", "skycube_dev_prefilter",
     "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
-    "skycube_ctx_info",
+    "skycube_ctx_info", "skycube_ctx_counters",
 )
 
 
@@ -92,9 +92,10 @@ def lib():
         L.skycube_ctx_launches.argtypes = [P]
         L.skycube_ctx_launches.restype = I64
         L.skycube_ctx_info.argtypes = [P, ctypes.POINTER(I64), ctypes.POINTER(U32), ctypes.POINTER(U32)]
+        L.skycube_ctx_counters.argtypes = [P, P]
         for f in ("skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
-                  "skycube_ctx_info"):
+                  "skycube_ctx_info", "skycube_ctx_counters"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -254,6 +255,12 @@ class Context:
     @property
     def launches(self) -> int:
         return lib().skycube_ctx_launches(self._h)
+
+    def counters(self) -> dict:
+        a = np.zeros(8, np.int64)
+        _check(lib().skycube_ctx_counters(self._h, a.ctypes.data_as(ctypes.c_void_p)))
+        return {"k1_box": int(a[0]), "k1_pair": int(a[1]), "k3_box": int(a[2]), "k3_pair": int(a[3]),
+                "k3_miss": int(a[4])}
 
     def info(self):
         m, W, ex = ctypes.c_int64(), ctypes.c_uint32(), ctypes.c_uint32()

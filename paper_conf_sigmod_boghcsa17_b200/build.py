@@ -15,13 +15,13 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-OBJ = os.path.join(PKG, "build")
-LIB = os.path.join(PKG, "libskycube.so")
+OBJ = os.path.join(PKG, "build" + os.environ.get("SKYCUBE_BUILD_SUFFIX", ""))
+LIB = os.path.join(PKG, "libskycube%s.so" % os.environ.get("SKYCUBE_BUILD_SUFFIX", ""))
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
-         "-I" + os.path.join(ROOT, "include")]
+         "-I" + os.path.join(ROOT, "include")] + os.environ.get("SKYCUBE_NVCC_EXTRA", "").split()
 
 
 def _sources():

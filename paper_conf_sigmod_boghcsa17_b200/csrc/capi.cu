@@ -107,6 +107,8 @@ skycube_ctx *new_ctx(int device) {
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
     x->c.num_sms = sms;
+    x->c.counters.ensure(sizeof(unsigned long long) * 8);
+    SKY_CUDA(cudaMemset(x->c.counters.p, 0, sizeof(unsigned long long) * 8));
     return x;
 }
 
@@ -294,13 +296,21 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
                            &c.counts, &c.scan_tmp, &c.flags, &c.scanned, &c.rbuf, &c.nanflag, &c.codes_id,
                            &c.codes_sorted, &c.ord_sorted, &c.ext_id_flag, &c.ext_idx, &c.key_flag, &c.key_idx,
                            &c.ext_ids, &c.p_codes, &c.p_ord, &c.q_codes, &c.q_ord, &c.tie, &c.lat_counts,
-                           &c.scan64_tmp, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
+                           &c.scan64_tmp, &c.chunks_all, &c.chunks_ext, &c.counters, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
                            &ctx->membership, &ctx->offsets, &ctx->ids})
         b->release();
     delete ctx;
 }
 
 int64_t skycube_ctx_launches(const skycube_ctx *ctx) { return ctx ? ctx->c.L.count : 0; }
+
+skycube_status skycube_ctx_counters(const skycube_ctx *ctx, int64_t *out8) {
+    if (!ctx || !out8) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        SKY_CUDA(cudaMemcpy(out8, ctx->c.counters.p, sizeof(int64_t) * 8, cudaMemcpyDeviceToHost));
+    });
+}
 
 skycube_status skycube_ctx_info(const skycube_ctx *ctx, int64_t *n_ext, uint32_t *words_per_row,
                                 uint32_t *exact_mask) {

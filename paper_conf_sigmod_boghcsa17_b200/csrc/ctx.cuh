@@ -67,8 +67,10 @@ struct Ctx {
     DevBuf tie;         // u32 tiled rows: tie contributions to B_{p notin S}
     DevBuf chunks_all;  // u32 [n/32][33][cw]  chunk records of all points (K1 competitors)
     DevBuf chunks_ext;  // u32 [m/32][33][cw]  chunk records of S+ (K3 competitors)
+    DevBuf chunk_keys, chunk_perm, q_codes_alt, q_ord_alt;  // chunk visiting order (strongest corner first)
     int64_t nchunks_all = 0, nchunks_ext = 0;
     DevBuf lat_counts;  // u64 [2^d * nchunks]
+    DevBuf counters;    // u64 [8]: K1 box tests, K1 pair tests, K3 box tests, K3 pair tests, K3 misses
     DevBuf scan64_tmp;
 };
 

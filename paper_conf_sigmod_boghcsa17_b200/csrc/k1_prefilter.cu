@@ -17,6 +17,8 @@
 #include "ctx.cuh"
 #include "tile_stream.cuh"
 
+#include <algorithm>
+
 namespace sky {
 namespace {
 
@@ -28,29 +30,29 @@ template <int CW>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
     const uint32_t *__restrict__ codes_sorted, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ ord_sorted, int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset,
-    int64_t blk_step, uint8_t *__restrict__ ext_sorted) {
+    int64_t blk_step, int tpc, uint8_t *__restrict__ ext_sorted, unsigned long long *__restrict__ counters) {
     constexpr int CWP = CW | 1;         // odd row stride: conflict-free per-lane task loads
     constexpr int REC = 33 * CW;        // chunk record words
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)(kWarps * REC)};
-    uint32_t *pH = smem + 4 * kStages + kStages * kWarps * REC;  // [kTasks][CWP]
-    uint32_t *domw = pH + kTasks * CWP;                           // [kTasks / 32] dominated bits
+    uint32_t *pH = smem + 4 * kStages + kStages * kWarps * REC;  // [tpc][CWP]
+    uint32_t *domw = pH + tpc * CWP;                              // [tpc / 32] dominated bits
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t blk = blk_offset + (int64_t)blockIdx.x * blk_step;
-    const int64_t s0 = blk * kTasks;
-    const int nt = (int)min((int64_t)kTasks, n - s0);
+    const int64_t s0 = blk * tpc;
+    const int nt = (int)min((int64_t)tpc, n - s0);
     const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
 
     if (threadIdx.x == 0) ring.init(kWarps);
-    for (int i = threadIdx.x; i < kTasks * CW; i += blockDim.x) {
+    for (int i = threadIdx.x; i < tpc * CW; i += blockDim.x) {
         const int t = i / CW, k = i % CW;
         uint32_t w = t < nt ? codes_sorted[(s0 + t) * CW + k] : 0u;
         if (2 * k >= d) w |= 0x00007fffu;      // padding dimensions never reject
         if (2 * k + 1 >= d) w |= 0x7fff0000u;
         pH[t * CWP + k] = w | kGuard;
     }
-    for (int i = threadIdx.x; i < kTasks / 32; i += blockDim.x) {
+    for (int i = threadIdx.x; i < tpc / 32; i += blockDim.x) {
         uint32_t dead = 0;  // tasks past n count as dominated
         for (int b = 0; b < 32; b++)
             if (i * 32 + b >= nt) dead |= 1u << b;
@@ -69,6 +71,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
     for (int k = 0; k < CW; k++)
         csub[k] = (((inexact >> (2 * k)) & 1u) ? 0u : 1u) | (((inexact >> (2 * k + 1)) & 1u) ? 0u : 0x10000u);
     const int ngroups = (nt + 31) >> 5;
+    unsigned long long n_box = 0, n_pair = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t *rec = ring.stage(tile) + warp * REC;
@@ -92,6 +95,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
             for (int k = 0; k < CW; k++) acc &= pH[tt * CWP + k] - mn[k] - csub[k];  // corner below p
             const bool cand = !((dw >> lane) & 1u) && (acc & kGuard) == kGuard;
             uint32_t need = __ballot_sync(0xffffffffu, cand);
+            n_box += __popc(~dw);
+            n_pair += 32u * __popc(need);
             while (need) {
                 const int b = __ffs(need) - 1;
                 need &= need - 1;
@@ -126,42 +131,54 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
             }
         }
     }
+    if (lane == 0 && counters) {
+        atomicAdd(&counters[0], n_box);
+        atomicAdd(&counters[1], n_pair);
+    }
     asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32) : "memory");
     for (int t = threadIdx.x; t < nt; t += kWarps * 32) ext_sorted[s0 + t] = ((domw[t >> 5] >> (t & 31)) & 1u) ? 0 : 1;
 }
 
 template <int CW>
-void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uint8_t *ext, cudaStream_t st) {
+void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, int tpc, uint8_t *ext, cudaStream_t st) {
     constexpr int CWP = CW | 1;
-    const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * kWarps * 33 * CW + (size_t)kTasks * CWP +
-                                            kTasks / 32);
+    const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * kWarps * 33 * CW + (size_t)tpc * CWP +
+                                            tpc / 32);
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
     k1_prefilter_kernel<CW><<<(unsigned)nblk_mine, (kWarps + 1) * 32, smem, st>>>(
         c.codes_sorted.as<uint32_t>(), c.chunks_all.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, inexact,
-        c.nchunks_all, blk_offset, blk_step, ext);
+        c.nchunks_all, blk_offset, blk_step, tpc, ext, c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
 
 }  // namespace
 
-// Blocks of kTasks consecutive tree positions; block b is processed iff b % tile_step == tile_offset.
+int prefilter_block_size(int64_t n, int64_t step);
+
+// Blocks of tpc consecutive tree positions; block b is processed iff b % tile_step == tile_offset.
 void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ext_sorted, cudaStream_t st) {
     if (!c.prepared) throw Error{1, "skycube_dev_prefilter before skycube_dev_prepare"};
     if (tile_step < 1 || tile_offset < 0) throw Error{1, "bad prefilter block range"};
-    const int64_t nblk = ceil_div(c.n, kTasks);
+    const int tpc = prefilter_block_size(c.n, tile_step);
+    const int64_t nblk = ceil_div(c.n, tpc);
     if (tile_offset >= nblk) return;
     const int64_t mine = (nblk - 1 - tile_offset) / tile_step + 1;
     switch (c.dp / 2) {
-        case 2: launch<2>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
-        case 4: launch<4>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
-        case 6: launch<6>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
-        case 8: launch<8>(c, tile_offset, tile_step, mine, d_ext_sorted, st); break;
+        case 2: launch<2>(c, tile_offset, tile_step, mine, tpc, d_ext_sorted, st); break;
+        case 4: launch<4>(c, tile_offset, tile_step, mine, tpc, d_ext_sorted, st); break;
+        case 6: launch<6>(c, tile_offset, tile_step, mine, tpc, d_ext_sorted, st); break;
+        case 8: launch<8>(c, tile_offset, tile_step, mine, tpc, d_ext_sorted, st); break;
         default: throw Error{1, "unsupported dimensionality"};
     }
 }
 
-int64_t prefilter_block_size() { return kTasks; }
+// Tasks per CTA: up to kTasks, but small enough that every rank (step = number of ranks) gets at least
+// two CTAs per SM.  Depends only on (n, step), so every rank derives the same blocks.
+int prefilter_block_size(int64_t n, int64_t step) {
+    const int64_t want = ceil_div(n, step * 2 * 148);
+    return (int)std::max<int64_t>(32, std::min<int64_t>(kTasks, ceil_div(want, 32) * 32));
+}
 
 }  // namespace sky

@@ -25,6 +25,7 @@
 //   design B (d > 12): a CTA holds the states of NT tasks (192 KB in total, 8 KB per task at d = 16);
 //     each lane holds one competitor in registers and runs it against all NT tasks (task codes are
 //     broadcasts); misses expand with shared-memory atomics.
+#include <algorithm>
 #include <cstdlib>
 
 #include "ctx.cuh"
@@ -363,15 +364,35 @@ __global__ void __launch_bounds__((kBWarps + 1) * 32, 1) k3_mdmc_b_kernel(
 //              shared-memory broadcast) and probes the task's state; misses run Alg. 3 lines 10-12 with
 //              shared-memory atomics (several warps may update one task).
 constexpr int kCWarps = 16;
-constexpr int kCStages = 3;
-constexpr int kCStateBytes = 144 * 1024;
+constexpr int kCStages = 4;
+constexpr int kCSmemBytes = 227 * 1024;  // opt-in maximum per CTA
 constexpr int kCU = 4;
+
+// CW words from a 16-byte aligned row (CW even): LDS.128 / LDS.64 instead of CW scalar loads.
+template <int CW>
+__device__ __forceinline__ void load_row(const uint32_t *p, uint32_t *w) {
+#pragma unroll
+    for (int k = 0; k + 4 <= CW; k += 4) {
+        const uint4 v = *reinterpret_cast<const uint4 *>(p + k);
+        w[k] = v.x;
+        w[k + 1] = v.y;
+        w[k + 2] = v.z;
+        w[k + 3] = v.w;
+    }
+    if (CW % 4) {
+        const uint2 v = *reinterpret_cast<const uint2 *>(p + (CW & ~3));
+        w[CW & ~3] = v.x;
+        w[(CW & ~3) + 1] = v.y;
+    }
+}
 
 template <int D, bool TIES>
 struct GeoC {
-    static constexpr int PER = (TIES ? 2 : 1) * Geo<D>::WB;       // state words per task
-    static constexpr int NT0 = kCStateBytes / (PER * 4);
-    static constexpr int NT = NT0 < 1024 ? NT0 : 1024;            // tasks per CTA
+    static constexpr int PER = (TIES ? 2 : 1) * Geo<D>::WB;                   // state words per task
+    static constexpr int ROW = PER + ((Geo<D>::CW + 3) & ~3) + (Geo<D>::CW | 1);  // words per task
+    static constexpr int RING = 4 * kCStages + kCStages * kCWarps * 33 * Geo<D>::CW;  // words
+    static constexpr int NT0 = (kCSmemBytes / 4 - RING - 128 - kCWarps * 64) / ROW;
+    static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                         // tasks per CTA
 };
 
 template <int D, bool TIES>
@@ -406,34 +427,84 @@ __device__ __forceinline__ void mdmc_miss_c(uint32_t *st, const uint32_t *ph, co
     } while (w);
 }
 
+// Exact B_{q<=p}, B_{q<p} from the guard-bit compares plus exact keys on tied, non-injective codes.
+template <int D>
+__device__ __forceinline__ void exact_masks(const uint32_t *ph, const uint32_t *q, uint32_t M, uint32_t inexact,
+                                            const uint32_t *__restrict__ qo, const uint32_t *__restrict__ po,
+                                            uint32_t &L, uint32_t &S) {
+    using G = Geo<D>;
+    uint32_t lt[G::CW];
+#pragma unroll
+    for (int k = 0; k < G::CW; k++) lt[k] = ph[k] - q[k] - 0x00010001u;
+    S = gather_mask<G::NG>(lt);
+    L = M;
+    const uint32_t U = M & ~S & inexact;
+    if (U) refine_exact(U, qo, po, L, S);
+}
+
+// Warp-cooperative word-parallel expansion: dst |= { delta subset of X : not delta subset of E } (E subset X);
+// E = 0 gives sub(X) (the empty set included, harmless: bit 0 is cleared on output).  Word w of dst at
+// dst[w * stride].  The lanes take the subsets of the lowest five word-index bits of X; every lane
+// iterates the subsets of the remaining word-index bits.  Atomic: other warps update the same task.
+__device__ __forceinline__ void coop_down_or(uint32_t *dst, int stride, uint32_t X, uint32_t E, int lane) {
+    const uint32_t xh = X >> 5, eh = E >> 5;
+    const uint32_t xb = sub5(X & 31u), eb = sub5(E & 31u);
+    uint32_t rest = xh, w_lo = 0;
+    int np = 0;
+#pragma unroll
+    for (int i = 0; i < 5; i++) {
+        if (rest) {
+            const uint32_t bit = rest & (0u - rest);
+            rest &= rest - 1;
+            if ((lane >> i) & 1) w_lo |= bit;
+            np++;
+        }
+    }
+    if (lane < (1 << np)) {
+        uint32_t w_hi = 0;
+        do {
+            const uint32_t w = w_lo | w_hi;
+            const uint32_t bits = (w & ~eh) ? xb : (xb & ~eb);
+            if (bits) atomicOr(&dst[w * stride], bits);
+            w_hi = (w_hi - rest) & rest;
+        } while (w_hi);
+    }
+    __syncwarp();
+}
+
 template <int D, bool TIES>
 __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
-    const uint32_t *__restrict__ q_ord, int64_t nchunks, int64_t j_begin, int64_t j_end, uint32_t inexact,
-    uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32) {
+    const uint32_t *__restrict__ q_ord, int64_t nchunks, int64_t j_begin, int64_t j_end, uint32_t inexact, int tpc,
+    uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32,
+    unsigned long long *__restrict__ counters) {
     using G = Geo<D>;
     using C = GeoC<D, TIES>;
-    constexpr int CWP = G::CW | 1;
+    constexpr int CWP = G::CW | 1;           // odd stride: per-lane row loads are conflict-free (box pass)
+    constexpr int CWV = (G::CW + 3) & ~3;    // 16-byte stride: broadcast vector loads (pair pass)
     constexpr int REC = 33 * G::CW;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     const TileRing<kCStages> ring{bars, bars + kCStages, smem + 4 * kCStages, (uint32_t)(kCWarps * REC)};
-    uint32_t *pH = smem + 4 * kCStages + kCStages * kCWarps * REC;  // [NT][CWP]
-    uint32_t *state = pH + C::NT * CWP;                              // [NT][PER]
+    uint32_t *pV = smem + 4 * kCStages + kCStages * kCWarps * REC;  // [tpc][CWV]
+    uint32_t *pH = pV + tpc * CWV;                                   // [tpc][CWP]
+    uint32_t *state = pH + tpc * CWP;                                // [tpc][PER]
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int64_t j0 = j_begin + (int64_t)blockIdx.x * C::NT;
-    const int nt = (int)min((int64_t)C::NT, j_end - j0);
+    uint32_t *mq = state + tpc * C::PER + warp * 64;                 // per-warp miss queue [32][2]
+    const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
+    const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, kCWarps);
 
     if (threadIdx.x == 0) ring.init(kCWarps);
-    for (int i = threadIdx.x; i < C::NT * G::CW; i += blockDim.x) {
+    for (int i = threadIdx.x; i < tpc * G::CW; i += blockDim.x) {
         const int t = i / G::CW, k = i % G::CW;
         uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
         if (2 * k >= D) w &= 0xffff0000u;  // padding dimensions: p = 0 never passes q <= p (q pad = 1)
         if (2 * k + 1 >= D) w &= 0x0000ffffu;
         pH[t * CWP + k] = w | kGuard;
+        pV[t * CWV + k] = w | kGuard;
     }
-    for (int i = threadIdx.x; i < C::NT * C::PER; i += blockDim.x) state[i] = (i % C::PER) == 0 ? 1u : 0u;
+    for (int i = threadIdx.x; i < tpc * C::PER; i += blockDim.x) state[i] = (i % C::PER) == 0 ? 1u : 0u;
     __syncthreads();
     if (warp == kCWarps) {
         if (lane == 0)
@@ -441,6 +512,7 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
         return;
     }
     const int ngroups = (nt + 31) >> 5;
+    unsigned long long n_box = 0, n_pair = 0, n_miss = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t *rec = ring.stage(tile) + warp * REC;
@@ -464,6 +536,8 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
             const uint32_t wb = state[tt * C::PER + (Mb >> 5)];
             const bool need = g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
             uint32_t todo = __ballot_sync(0xffffffffu, need);
+            n_box += min(32, nt - g * 32);
+            n_pair += 32u * __popc(todo);
             while (todo) {
                 int ts[kCU];
                 int cnt = 0;
@@ -478,10 +552,10 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
                 uint32_t M[kCU], wd[kCU];
 #pragma unroll
                 for (int u = 0; u < kCU; u++) {
-                    const uint32_t *ph = pH + ts[u] * CWP;
                     uint32_t x[G::CW];
+                    load_row<G::CW>(pV + ts[u] * CWV, x);
 #pragma unroll
-                    for (int k = 0; k < G::CW; k++) x[k] = ph[k] - q[k];
+                    for (int k = 0; k < G::CW; k++) x[k] -= q[k];
                     M[u] = gather_mask<G::NG>(x);
                     wd[u] = state[ts[u] * C::PER + (M[u] >> 5)];
                 }
@@ -493,14 +567,54 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
                 for (int u = 0; u < kCU; u++) {
                     if (u >= cnt) break;
                     uint32_t *st = state + ts[u] * C::PER;
-                    if ((st[M[u] >> 5] >> (M[u] & 31)) & 1u) continue;
                     const int64_t jt = j0 + ts[u];
+#ifndef SKY_COOP_MISS
+                    if ((st[M[u] >> 5] >> (M[u] & 31)) & 1u) continue;
+                    n_miss++;
                     uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
                     mdmc_miss_c<D, TIES>(st, pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D,
                                          tr, TIES ? 1 : 32);
+#else
+                    // lane-local exact masks for the lanes that missed (Alg. 3 lines 10-11)
+                    uint32_t L = 0, S = 0;
+                    if (!((st[M[u] >> 5] >> (M[u] & 31)) & 1u)) {
+                        n_miss++;
+                        exact_masks<D>(pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D, L, S);
+                        if (L != M[u] && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;
+                    }
+                    // line 12, warp-cooperative: contributing competitors are queued in shared memory (explicit
+                    // reconvergence, no shuffles in divergent code), then all lanes expand each one
+                    const uint32_t todo_m = __ballot_sync(0xffffffffu, S != 0);
+                    if (S != 0) {
+                        const int slot = __popc(todo_m & ((1u << lane) - 1u));
+                        mq[2 * slot] = S;
+                        mq[2 * slot + 1] = L;
+                    }
+                    __syncwarp();
+                    const int nq = __popc(todo_m);
+                    for (int e = 0; e < nq; e++) {
+                        const uint32_t Sb = mq[2 * e], Lb = mq[2 * e + 1];
+                        const uint32_t sw = st[Sb >> 5];
+                        __syncwarp();
+                        if (!((sw >> (Sb & 31)) & 1u)) coop_down_or(st, 1, Sb, 0u, lane);
+                        if (Lb != Sb) {
+                            uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+                            coop_down_or(tr, TIES ? 1 : 32, Lb, Lb & ~Sb, lane);
+                        }
+                    }
+                    __syncwarp();
+#endif
                 }
             }
         }
+    }
+    if (counters) {
+        if (lane == 0) {
+            atomicAdd(&counters[2], n_box);
+            atomicAdd(&counters[3], n_pair);
+        }
+        for (int o = 16; o; o >>= 1) n_miss += __shfl_xor_sync(0xffffffffu, n_miss, o);
+        if (lane == 0) atomicAdd(&counters[4], n_miss);
     }
     asm volatile("bar.sync 1, %0;" ::"r"(kCWarps * 32) : "memory");
     for (int t = warp; t < nt; t += kCWarps) {
@@ -526,13 +640,18 @@ template <int D, bool TIES>
 void launch_c_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
     using C = GeoC<D, TIES>;
+    // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
+    const int64_t range = j_end - j_begin;
+    const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
     const size_t smem = sizeof(uint32_t) * (4 * kCStages + (size_t)kCStages * kCWarps * 33 * G::CW +
-                                            (size_t)C::NT * (G::CW | 1) + (size_t)C::NT * C::PER);
+                                            (size_t)tpc * (((G::CW + 3) & ~3) + (G::CW | 1)) + (size_t)tpc * C::PER +
+                                            kCWarps * 64);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_c_kernel<D, TIES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    const unsigned blocks = (unsigned)ceil_div(j_end - j_begin, C::NT);
+    const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_mdmc_c_kernel<D, TIES><<<blocks, (kCWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), rows32, c.tie.as<uint32_t>(), ext_rows32);
+        c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc, rows32, c.tie.as<uint32_t>(), ext_rows32,
+        c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }

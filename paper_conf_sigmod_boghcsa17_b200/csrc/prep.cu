@@ -14,6 +14,8 @@
 // bit 2 the quartile split, ... (L338 "median, then quartile, then octile").  Consecutive runs of 32
 // points in that order are "chunks" whose per-dimension minimum codes bound every member; K1 and K3
 // test a whole chunk against a task with one mask test (Eq. 1's idea, L1312) before any pair.
+#include <utility>
+
 #include "ctx.cuh"
 
 namespace sky {
@@ -170,6 +172,29 @@ __global__ void ext_build_key_kernel(const uint32_t *__restrict__ key_flag, cons
 
 inline unsigned blocks_for(int64_t n, int t) { return (unsigned)ceil_div(n > 0 ? n : 1, t); }
 
+// key of a chunk = sum of its lower-corner codes (< 2^20 for d <= 16)
+__global__ void chunk_key_kernel(const uint32_t *__restrict__ chunks, int64_t nch, int cw, int d,
+                                 uint64_t *__restrict__ keys, uint32_t *__restrict__ perm) {
+    const int64_t ch = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (ch >= nch) return;
+    const uint32_t *mn = chunks + ch * (int64_t)(33 * cw) + 32 * cw;
+    uint64_t s = 0;
+    for (int i = 0; i < d; i++) s += (mn[i >> 1] >> (16 * (i & 1))) & 0xffffu;
+    keys[ch] = s;
+    perm[ch] = (uint32_t)ch;
+}
+
+// point j of new chunk c' <- point j of old chunk perm[c'] (codes and exact keys)
+__global__ void permute_chunks_kernel(const uint32_t *__restrict__ perm, int64_t nch, int cw, int d,
+                                      const uint32_t *__restrict__ codes, const uint32_t *__restrict__ ord,
+                                      uint32_t *__restrict__ codes_out, uint32_t *__restrict__ ord_out) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nch * 32) return;
+    const int64_t src = (int64_t)perm[i >> 5] * 32 + (i & 31);
+    for (int k = 0; k < cw; k++) codes_out[i * cw + k] = codes[src * cw + k];
+    for (int k = 0; k < d; k++) ord_out[i * d + k] = ord[src * d + k];
+}
+
 __global__ void fill_kernel(uint32_t *a, int64_t from, int64_t to, uint32_t v) {
     const int64_t i = from + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < to) a[i] = v;
@@ -323,11 +348,38 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     SKY_LAUNCH_CHECK();
     pad_codes(c.q_codes.as<uint32_t>(), m, mpad, cw, st, c.L);
     pad_ord(c.q_ord.as<uint32_t>(), m, mpad, d, st, c.L);
+    // Chunks of the static-tree order, then visited strongest lower corner first (smallest sum of corner
+    // codes): B_{p notin S+} saturates early, so later chunks resolve by their corner test.
+    const int64_t nch = ceil_div(m, 32);
+    c.chunk_keys.ensure(sizeof(uint64_t) * nch);
+    c.chunk_perm.ensure(sizeof(uint32_t) * nch);
+    c.q_codes_alt.ensure(sizeof(uint32_t) * mpad * cw);
+    c.q_ord_alt.ensure(sizeof(uint32_t) * mpad * d);
     build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw,
                                                               c.chunks_ext.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
-    c.nchunks_ext = ceil_div(m, 32);
+    chunk_key_kernel<<<blocks_for(nch, 256), 256, 0, st>>>(c.chunks_ext.as<uint32_t>(), nch, cw, d,
+                                                           c.chunk_keys.as<uint64_t>(), c.chunk_perm.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    radix_sort_u64(c.chunk_keys.as<uint64_t>(), c.chunk_perm.as<uint32_t>(), nch, 20, c.keys_alt.as<uint64_t>(),
+                   c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
+    permute_chunks_kernel<<<blocks_for(nch * 32, 256), 256, 0, st>>>(c.chunk_perm.as<uint32_t>(), nch, cw, d,
+                                                                     c.q_codes.as<uint32_t>(), c.q_ord.as<uint32_t>(),
+                                                                     c.q_codes_alt.as<uint32_t>(),
+                                                                     c.q_ord_alt.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    std::swap(c.q_codes, c.q_codes_alt);
+    std::swap(c.q_ord, c.q_ord_alt);
+    pad_codes(c.q_codes.as<uint32_t>(), nch * 32, mpad, cw, st, c.L);
+    pad_ord(c.q_ord.as<uint32_t>(), nch * 32, mpad, d, st, c.L);
+    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw,
+                                                              c.chunks_ext.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    c.nchunks_ext = nch;
     c.ext_ready = true;
 }
 

@@ -43,6 +43,24 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     } while (!done);
 }
 
+// Producer-side wait: back off with nanosleep between probes so that a waiting producer warp does not
+// steal issue slots from the consumer warps of its SM sub-partition.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+    const uint32_t addr = smem_u32(bar);
+    uint32_t done;
+    uint32_t ns = 32;
+    while (true) {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(addr), "r"(parity)
+            : "memory");
+        if (done) return;
+        __nanosleep(ns);
+        ns = ns < 1024 ? ns * 2 : ns;
+    }
+}
+
 // Double-buffered stream of fixed-size tiles (bytes multiple of 16, 16-B aligned source).
 struct TileStream2 {
     uint64_t *bar;  // [2] in shared memory
@@ -90,7 +108,7 @@ struct TileRing {
     }
     __device__ __forceinline__ void issue(const uint32_t *src_tiles, int64_t t) const {
         const int s = (int)(t % S);
-        if (t >= S) mbar_wait(&empty[s], (uint32_t)(((t / S) - 1) & 1));
+        if (t >= S) mbar_wait_sleep(&empty[s], (uint32_t)(((t / S) - 1) & 1));
         const uint32_t bytes = tile_words * 4u;
         mbar_arrive_expect_tx(&full[s], bytes);
         bulk_g2s(buf + (uint32_t)s * tile_words, src_tiles + t * (int64_t)tile_words, bytes, &full[s]);
