@@ -210,7 +210,10 @@ def run_ours(args):
     def step(events=None):
         return eng.build(pts, lists=True, membership=True, events=events)
 
+    out = None
     for _ in range(args.warmup):
+        out = step()
+    if out is None:  # --warmup 0 (profiling runs): one untimed build still fixes n_ext and the id count
         out = step()
     torch.cuda.synchronize()
     m = out["n_ext"]
