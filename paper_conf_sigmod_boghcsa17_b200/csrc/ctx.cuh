@@ -53,6 +53,7 @@ struct Ctx {
     DevBuf flags;       // u32 [n*d]
     DevBuf scanned;     // u32 [n*d]
     DevBuf rbuf;        // u32 [kMaxD]
+    DevBuf minord;      // u32 [kMaxD]  key of each dimension's minimum value
     DevBuf nanflag;     // u32 [1]
     DevBuf codes_id;    // u16 [n*dp]  id order
     DevBuf codes_sorted;// u16 [npad*dp]  static-tree (Morton) order, padded to whole chunk tiles
@@ -68,6 +69,7 @@ struct Ctx {
     DevBuf chunks_all;  // u32 [n/32][33][cw]  chunk records of all points (K1 competitors)
     DevBuf chunks_ext;  // u32 [m/32][33][cw]  chunk records of S+ (K3 competitors)
     DevBuf chunk_keys, chunk_perm, q_codes_alt, q_ord_alt;  // chunk visiting order (strongest corner first)
+    DevBuf supers_all, supers_ext;  // u32 [tiles][super_words(cw)]  lower corner of each tile of 16 chunks
     int64_t nchunks_all = 0, nchunks_ext = 0;
     DevBuf lat_counts;  // u64 [2^d * nchunks]
     DevBuf counters;    // u64 [8]: K1 box tests, K1 pair tests, K3 box tests, K3 pair tests, K3 misses
@@ -89,5 +91,7 @@ void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *
 constexpr int kPrefilterTile = 256;  // sorted positions per K1 block
 constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
 constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole
+constexpr int kTileChunks = 16;         // chunks per competitor tile (one super-chunk of 512 points)
+inline int super_words(int cw) { return (cw + 3) & ~3; }  // super-corner record words (16-byte multiple)
 
 }  // namespace sky

@@ -22,32 +22,35 @@
 namespace sky {
 namespace {
 
-constexpr int kWarps = 16;         // consumer warps = chunks per tile
+constexpr int kWarps = kTileChunks;  // consumer warps = chunks per tile
 constexpr int kTasks = 2048;       // tasks per CTA
 constexpr int kStages = 3;
 
 template <int CW>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
-    const uint32_t *__restrict__ codes_sorted, const uint32_t *__restrict__ chunks,
-    const uint32_t *__restrict__ ord_sorted, int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset,
-    int64_t blk_step, int tpc, uint8_t *__restrict__ ext_sorted, unsigned long long *__restrict__ counters) {
+    const uint32_t *__restrict__ chunks, const uint32_t *__restrict__ supers, const uint32_t *__restrict__ ord_sorted,
+    int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset, int64_t blk_step, int tpc,
+    uint8_t *__restrict__ ext_sorted, unsigned long long *__restrict__ counters) {
     constexpr int CWP = CW | 1;         // odd row stride: conflict-free per-lane task loads
     constexpr int REC = 33 * CW;        // chunk record words
+    constexpr int CWS = (CW + 3) & ~3;  // super-corner record words
+    constexpr int TW = kTileChunks * REC + CWS;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
-    const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)(kWarps * REC)};
-    uint32_t *pH = smem + 4 * kStages + kStages * kWarps * REC;  // [tpc][CWP]
+    const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)TW};
+    uint32_t *pH = smem + 4 * kStages + kStages * TW;             // [tpc][CWP]
     uint32_t *domw = pH + tpc * CWP;                              // [tpc / 32] dominated bits
+    uint32_t *needw = domw + tpc / 32;                            // [2][tpc / 32] tasks below the tile corner
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t blk = blk_offset + (int64_t)blockIdx.x * blk_step;
     const int64_t s0 = blk * tpc;
     const int nt = (int)min((int64_t)tpc, n - s0);
-    const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
+    const int64_t ntiles = ceil_div_dev(nchunks, kTileChunks);
 
     if (threadIdx.x == 0) ring.init(kWarps);
     for (int i = threadIdx.x; i < tpc * CW; i += blockDim.x) {
         const int t = i / CW, k = i % CW;
-        uint32_t w = t < nt ? codes_sorted[(s0 + t) * CW + k] : 0u;
+        uint32_t w = t < nt ? chunks[((s0 + t) >> 5) * REC + ((s0 + t) & 31) * CW + k] : 0u;
         if (2 * k >= d) w |= 0x00007fffu;      // padding dimensions never reject
         if (2 * k + 1 >= d) w |= 0x7fff0000u;
         pH[t * CWP + k] = w | kGuard;
@@ -61,7 +64,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
     __syncthreads();
     if (warp == kWarps) {
         if (lane == 0)
-            for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
+            for (int64_t t = 0; t < ntiles; t++) ring.issue2(chunks, kTileChunks * REC, supers, CWS, t);
         return;
     }
     // corner test: q < p needs code(q) < code(p) on injective dimensions but only code(q) <= code(p) on
@@ -74,32 +77,55 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
     unsigned long long n_box = 0, n_pair = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
-        const uint32_t *rec = ring.stage(tile) + warp * REC;
+        const uint32_t *stg = ring.stage(tile);
+        uint32_t *need = needw + (tile & 1) * (tpc / 32);
+        // phase A (super-chunk test, the upper level of the static tree): which live tasks lie strictly above
+        // the tile's lower corner; groups of 32 tasks are spread over the warps
+        {
+            uint32_t sc[CW];
+#pragma unroll
+            for (int k = 0; k < CW; k++) sc[k] = stg[kTileChunks * REC + k] + csub[k];
+            for (int g = warp; g < ngroups; g += kWarps) {
+                const uint32_t dw = domw[g];
+                uint32_t nb = 0;
+                if (dw != 0xffffffffu) {
+                    const int tt = g * 32 + lane;
+                    uint32_t acc = 0xffffffffu;
+#pragma unroll
+                    for (int k = 0; k < CW; k++) acc &= pH[tt * CWP + k] - sc[k];
+                    nb = __ballot_sync(0xffffffffu, !((dw >> lane) & 1u) && (acc & kGuard) == kGuard);
+                    n_box += __popc(~dw);
+                }
+                if (lane == 0) need[g] = nb;
+            }
+        }
+        consumer_sync(kWarps * 32);
+        // phase B: one chunk per warp, only for the tasks of phase A
+        const uint32_t *rec = stg + warp * REC;
         uint32_t q[CW], mn[CW];
 #pragma unroll
         for (int k = 0; k < CW; k++) {
             q[k] = rec[lane * CW + k];
-            mn[k] = rec[32 * CW + k];
+            mn[k] = rec[32 * CW + k] + csub[k];
         }
         __syncwarp();
         if (lane == 0) ring.release(tile);
-        const int64_t c = tile * kWarps + warp;
+        const int64_t c = tile * kTileChunks + warp;
         if (c >= nchunks) continue;
         const int64_t qpos = c * 32 + lane;
         for (int g = 0; g < ngroups; g++) {
+            const uint32_t nw = need[g] & ~domw[g];
+            if (nw == 0) continue;
             const int tt = g * 32 + lane;
-            const uint32_t dw = domw[g];
-            if (dw == 0xffffffffu) continue;
             uint32_t acc = 0xffffffffu;
 #pragma unroll
-            for (int k = 0; k < CW; k++) acc &= pH[tt * CWP + k] - mn[k] - csub[k];  // corner below p
-            const bool cand = !((dw >> lane) & 1u) && (acc & kGuard) == kGuard;
-            uint32_t need = __ballot_sync(0xffffffffu, cand);
-            n_box += __popc(~dw);
-            n_pair += 32u * __popc(need);
-            while (need) {
-                const int b = __ffs(need) - 1;
-                need &= need - 1;
+            for (int k = 0; k < CW; k++) acc &= pH[tt * CWP + k] - mn[k];  // chunk corner below p
+            uint32_t todo = __ballot_sync(0xffffffffu, ((nw >> lane) & 1u) && (acc & kGuard) == kGuard);
+            n_box += __popc(nw);
+            n_pair += 32u * __popc(todo);
+            while (todo) {
+                const int b = __ffs(todo) - 1;
+                todo &= todo - 1;
                 const int ts = g * 32 + b;
                 const uint32_t *ph = pH + ts * CWP;
                 uint32_t lt = 0xffffffffu, le = 0xffffffffu;
@@ -135,19 +161,19 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
         atomicAdd(&counters[0], n_box);
         atomicAdd(&counters[1], n_pair);
     }
-    asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32) : "memory");
+    consumer_sync(kWarps * 32);
     for (int t = threadIdx.x; t < nt; t += kWarps * 32) ext_sorted[s0 + t] = ((domw[t >> 5] >> (t & 31)) & 1u) ? 0 : 1;
 }
 
 template <int CW>
 void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, int tpc, uint8_t *ext, cudaStream_t st) {
     constexpr int CWP = CW | 1;
-    const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * kWarps * 33 * CW + (size_t)tpc * CWP +
-                                            tpc / 32);
+    const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * (kTileChunks * 33 * CW + ((CW + 3) & ~3)) +
+                                            (size_t)tpc * CWP + 3 * (tpc / 32));
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
     k1_prefilter_kernel<CW><<<(unsigned)nblk_mine, (kWarps + 1) * 32, smem, st>>>(
-        c.codes_sorted.as<uint32_t>(), c.chunks_all.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, inexact,
+        c.chunks_all.as<uint32_t>(), c.supers_all.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, inexact,
         c.nchunks_all, blk_offset, blk_step, tpc, ext, c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();

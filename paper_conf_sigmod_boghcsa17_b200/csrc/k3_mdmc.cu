@@ -386,16 +386,30 @@ __device__ __forceinline__ void load_row(const uint32_t *p, uint32_t *w) {
     }
 }
 
-template <int D, bool TIES>
+// State modes of design C (per task, in shared memory):
+//   kModeGlobalTie  B_{p notin S+} (the probe set); the tie part of B_{p notin S} in a global row (continuous data)
+//   kModeSmemTie    B_{p notin S+} and the tie part, both in shared memory
+//   kModeDims       tie-exact state (reading Q3/Q4 made cheap under heavy ties): one downward-closed set per
+//                   dimension, D_i = union of sub(L_q) over the q with i in S_q, and the probe set
+//                   K = { delta : delta in D_i for every i in delta \ Z_p } (Z_p: dimensions where p holds the
+//                   global minimum, so no q is strictly better there).  p is dominated in delta <=> delta in D_i
+//                   for some i in delta (Def. 1: delta subset of L_q and delta & S_q != 0), and bit M in K proves
+//                   that q (S_q subset of L_q \ Z_p, L_q subset of M) adds nothing to any D_i.  Without ties K is
+//                   B_{p notin S+}; with ties K keeps growing where B_{p notin S+} cannot (ties at the optimum).
+constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
+
+template <int D, int MODE>
 struct GeoC {
-    static constexpr int PER = (TIES ? 2 : 1) * Geo<D>::WB;                   // state words per task
-    static constexpr int ROW = PER + ((Geo<D>::CW + 3) & ~3) + (Geo<D>::CW | 1);  // words per task
-    static constexpr int RING = 4 * kCStages + kCStages * kCWarps * 33 * Geo<D>::CW;  // words
-    static constexpr int NT0 = (kCSmemBytes / 4 - RING - 128 - kCWarps * 64) / ROW;
+    static constexpr int PER = (MODE == kModeGlobalTie ? 1 : MODE == kModeSmemTie ? 2 : D + 1) * Geo<D>::WB;
+    static constexpr int PS = PER | 1;  // odd task stride: equal word indices of 32 tasks hit 32 banks
+    static constexpr int ROW = PS + ((Geo<D>::CW + 3) & ~3) + (Geo<D>::CW | 1);  // words per task
+    static constexpr int TW = kCWarps * 33 * Geo<D>::CW + ((Geo<D>::CW + 3) & ~3);  // tile: 16 chunks + super corner
+    static constexpr int RING = 4 * kCStages + kCStages * TW;  // words
+    static constexpr int NT0 = (kCSmemBytes / 4 - RING - 128 - kCWarps * 64) / (ROW + 1 + 1);
     static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                         // tasks per CTA
 };
 
-template <int D, bool TIES>
+template <int D>
 __device__ __forceinline__ void mdmc_miss_c(uint32_t *st, const uint32_t *ph, const uint32_t *q, uint32_t M,
                                             uint32_t inexact, const uint32_t *__restrict__ qo,
                                             const uint32_t *__restrict__ po, uint32_t *tr, int tstride) {
@@ -423,6 +437,57 @@ __device__ __forceinline__ void mdmc_miss_c(uint32_t *st, const uint32_t *ph, co
     uint32_t w = 0;
     do {
         atomicOr(&tr[w * tstride], (w & ~eh) ? lb : (lb & ~eb));
+        w = (w - lh) & lh;
+    } while (w);
+}
+
+// Exact B_{q<=p}, B_{q<p} from the guard-bit compares plus exact keys on tied, non-injective codes.
+template <int D>
+__device__ __forceinline__ void exact_masks(const uint32_t *ph, const uint32_t *q, uint32_t M, uint32_t inexact,
+                                            const uint32_t *__restrict__ qo, const uint32_t *__restrict__ po,
+                                            uint32_t &L, uint32_t &S);
+
+// Word pattern of the low-5-bit subspaces that contain dimension i (i < 5).
+__device__ __forceinline__ uint32_t low_dim_pattern(int i) {
+    return i == 0 ? 0xaaaaaaaau : i == 1 ? 0xccccccccu : i == 2 ? 0xf0f0f0f0u : i == 3 ? 0xff00ff00u : 0xffff0000u;
+}
+
+// kModeDims miss path (Alg. 3 lines 10-12 on the per-dimension sets).  st = [K | D_0 | ... | D_{d-1}].
+template <int D>
+__device__ __forceinline__ void mdmc_miss_dims(uint32_t *st, const uint32_t *ph, const uint32_t *q, uint32_t M,
+                                               uint32_t inexact, const uint32_t *__restrict__ qo,
+                                               const uint32_t *__restrict__ po, uint32_t z) {
+    using G = Geo<D>;
+    uint32_t L, S;
+    exact_masks<D>(ph, q, M, inexact, qo, po, L, S);
+    if (S == 0) return;                                              // q is nowhere better than p
+    if (L != M && ((st[L >> 5] >> (L & 31)) & 1u)) return;           // exact L already covered by K
+    const uint32_t lh = L >> 5, lb = sub5(L & 31u);
+    bool changed = false;
+    for (uint32_t s = S; s; s &= s - 1) {                            // D_i |= sub(L) for every i in S
+        uint32_t *Di = st + (1 + (__ffs(s) - 1)) * G::WB;
+        if ((Di[lh] >> (L & 31)) & 1u) continue;                     // downward closed: sub(L) already there
+        changed = true;
+        uint32_t w = 0;
+        do {
+            atomicOr(&Di[w], lb);
+            w = (w - lh) & lh;
+        } while (w);
+    }
+    if (!changed) return;
+    // K on the words of sub(L) (only there can D change).  Racing warps may compute K from stale D words:
+    // that only leaves K smaller (still sound); bits are only ever OR-ed in.
+    const volatile uint32_t *vs = st;
+    uint32_t w = 0;
+    do {
+        uint32_t k = 0xffffffffu;
+#pragma unroll
+        for (int i = 0; i < D; i++) {
+            if ((z >> i) & 1u) continue;
+            const uint32_t in = i < 5 ? low_dim_pattern(i) : (((w >> (i - 5)) & 1u) ? 0xffffffffu : 0u);
+            k &= vs[(1 + i) * G::WB + w] | ~in;
+        }
+        atomicOr(&st[w], k);
         w = (w - lh) & lh;
     } while (w);
 }
@@ -472,25 +537,30 @@ __device__ __forceinline__ void coop_down_or(uint32_t *dst, int stride, uint32_t
     __syncwarp();
 }
 
-template <int D, bool TIES>
+template <int D, int MODE>
 __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
-    const uint32_t *__restrict__ q_ord, int64_t nchunks, int64_t j_begin, int64_t j_end, uint32_t inexact, int tpc,
+    const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, const uint32_t *__restrict__ supers,
+    int use_super, int64_t nchunks, int64_t j_begin, int64_t j_end, uint32_t inexact, int tpc,
     uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32,
     unsigned long long *__restrict__ counters) {
     using G = Geo<D>;
-    using C = GeoC<D, TIES>;
+    using C = GeoC<D, MODE>;
+    constexpr bool TIES = MODE == kModeSmemTie;
     constexpr int CWP = G::CW | 1;           // odd stride: per-lane row loads are conflict-free (box pass)
     constexpr int CWV = (G::CW + 3) & ~3;    // 16-byte stride: broadcast vector loads (pair pass)
     constexpr int REC = 33 * G::CW;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
-    const TileRing<kCStages> ring{bars, bars + kCStages, smem + 4 * kCStages, (uint32_t)(kCWarps * REC)};
-    uint32_t *pV = smem + 4 * kCStages + kCStages * kCWarps * REC;  // [tpc][CWV]
+    const TileRing<kCStages> ring{bars, bars + kCStages, smem + 4 * kCStages, (uint32_t)C::TW};
+    uint32_t *pV = smem + 4 * kCStages + kCStages * C::TW;          // [tpc][CWV]
     uint32_t *pH = pV + tpc * CWV;                                   // [tpc][CWP]
     uint32_t *state = pH + tpc * CWP;                                // [tpc][PER]
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    uint32_t *mq = state + tpc * C::PER + warp * 64;                 // per-warp miss queue [32][2]
+    uint32_t *zm = state + tpc * C::PS;                             // [tpc] Z_p (kModeDims)
+    const int TG = (tpc + 31) >> 5;
+    uint32_t *needw = zm + tpc;                                      // [2][TG] tasks below the tile corner
+    uint32_t *mq = needw + 2 * TG + warp * 64;                       // per-warp miss queue [32][2]
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, kCWarps);
@@ -504,17 +574,54 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
         pH[t * CWP + k] = w | kGuard;
         pV[t * CWV + k] = w | kGuard;
     }
-    for (int i = threadIdx.x; i < tpc * C::PER; i += blockDim.x) state[i] = (i % C::PER) == 0 ? 1u : 0u;
+    if (MODE == kModeDims) {
+        // Z_p = { i : p[i] is the minimum of dimension i } (exact keys); K starts as sub(Z_p)
+        for (int t = threadIdx.x; t < tpc; t += blockDim.x) {
+            uint32_t z = 0;
+            if (t < nt)
+                for (int i = 0; i < D; i++)
+                    if (p_ord[(j0 + t) * D + i] == minord[i]) z |= 1u << i;
+            zm[t] = z;
+        }
+        __syncthreads();
+        for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) {
+            const int t = i / C::PS, w = i % C::PS;
+            const uint32_t z = zm[t], zh = z >> 5;
+            state[i] = w < G::WB && (w & ~zh) == 0 ? sub5(z & 31u) : 0u;
+        }
+    } else {
+        for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) state[i] = (i % C::PS) == 0 ? 1u : 0u;
+    }
     __syncthreads();
     if (warp == kCWarps) {
         if (lane == 0)
-            for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
+            for (int64_t t = 0; t < ntiles; t++) ring.issue2(chunks, kCWarps * REC, supers, (G::CW + 3) & ~3, t);
         return;
     }
     const int ngroups = (nt + 31) >> 5;
     unsigned long long n_box = 0, n_pair = 0, n_miss = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
+        uint32_t *need = needw + (tile & 1) * TG;
+        if (use_super) {
+            // phase A (upper level of the static tree): tasks whose B_{p notin S+} (or K) already holds the mask
+            // of the tile's lower corner skip all 16 chunks of the tile (Λ4 on 512 competitors at once)
+            uint32_t sc[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) sc[k] = ring.stage(tile)[kCWarps * REC + k];
+            for (int g = warp; g < ngroups; g += kCWarps) {
+                const int tt = min(g * 32 + lane, nt - 1);
+                uint32_t le[G::CW];
+#pragma unroll
+                for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - sc[k];
+                const uint32_t Ms = gather_mask<G::NG>(le);
+                const uint32_t ws = state[tt * C::PS + (Ms >> 5)];
+                const uint32_t nb = __ballot_sync(0xffffffffu, g * 32 + lane < nt && !(__funnelshift_r(ws, ws, Ms) & 1u));
+                if (lane == 0) need[g] = nb;
+                n_box += min(32, nt - g * 32);
+            }
+            consumer_sync(kCWarps * 32);
+        }
         const uint32_t *rec = ring.stage(tile) + warp * REC;
         uint32_t q[G::CW], mn[G::CW];
 #pragma unroll
@@ -528,15 +635,17 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
         if (c >= nchunks) continue;
         const int64_t qpos = c * 32 + lane;
         for (int g = 0; g < ngroups; g++) {
+            const uint32_t nw = use_super ? need[g] : 0xffffffffu;
+            if (nw == 0) continue;
             const int tt = min(g * 32 + lane, nt - 1);
             uint32_t le[G::CW];
 #pragma unroll
             for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
             const uint32_t Mb = gather_mask<G::NG>(le);
-            const uint32_t wb = state[tt * C::PER + (Mb >> 5)];
-            const bool need = g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
-            uint32_t todo = __ballot_sync(0xffffffffu, need);
-            n_box += min(32, nt - g * 32);
+            const uint32_t wb = state[tt * C::PS + (Mb >> 5)];
+            const bool needp = ((nw >> lane) & 1u) && g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
+            uint32_t todo = __ballot_sync(0xffffffffu, needp);
+            n_box += use_super ? __popc(nw) : min(32, nt - g * 32);
             n_pair += 32u * __popc(todo);
             while (todo) {
                 int ts[kCU];
@@ -557,7 +666,7 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
 #pragma unroll
                     for (int k = 0; k < G::CW; k++) x[k] -= q[k];
                     M[u] = gather_mask<G::NG>(x);
-                    wd[u] = state[ts[u] * C::PER + (M[u] >> 5)];
+                    wd[u] = state[ts[u] * C::PS + (M[u] >> 5)];
                 }
                 uint32_t hit = 0xffffffffu;
 #pragma unroll
@@ -566,14 +675,19 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
 #pragma unroll
                 for (int u = 0; u < kCU; u++) {
                     if (u >= cnt) break;
-                    uint32_t *st = state + ts[u] * C::PER;
+                    uint32_t *st = state + ts[u] * C::PS;
                     const int64_t jt = j0 + ts[u];
 #ifndef SKY_COOP_MISS
                     if ((st[M[u] >> 5] >> (M[u] & 31)) & 1u) continue;
                     n_miss++;
-                    uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-                    mdmc_miss_c<D, TIES>(st, pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D,
-                                         tr, TIES ? 1 : 32);
+                    if (MODE == kModeDims) {
+                        mdmc_miss_dims<D>(st, pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D,
+                                          zm[ts[u]]);
+                    } else {
+                        uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+                        mdmc_miss_c<D>(st, pH + ts[u] * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + jt * D, tr,
+                                       TIES ? 1 : 32);
+                    }
 #else
                     // lane-local exact masks for the lanes that missed (Alg. 3 lines 10-11)
                     uint32_t L = 0, S = 0;
@@ -619,11 +733,21 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
     asm volatile("bar.sync 1, %0;" ::"r"(kCWarps * 32) : "memory");
     for (int t = warp; t < nt; t += kCWarps) {
         const int64_t jt = j0 + t;
-        const uint32_t *st = state + t * C::PER;
+        const uint32_t *st = state + t * C::PS;
         uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
         const uint32_t *trg = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
         for (int w = lane; w < G::WB; w += 32) {
-            const uint32_t v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+            uint32_t v;
+            if (MODE == kModeDims) {  // p dominated in delta <=> delta in D_i for some i in delta
+                v = 0;
+#pragma unroll
+                for (int i = 0; i < D; i++) {
+                    const uint32_t in = i < 5 ? low_dim_pattern(i) : (((w >> (i - 5)) & 1u) ? 0xffffffffu : 0u);
+                    v |= st[(1 + i) * G::WB + w] & in;
+                }
+            } else {
+                v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+            }
             uint32_t row = ~v & G::kRowMask;
             if (w == 0) row &= ~1u;
             out[w * 32] = row;
@@ -636,31 +760,53 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
     }
 }
 
-template <int D, bool TIES>
+// Super-chunk (tile corner) phase of design C: off by default — on the anticorrelated workloads the tile
+// corner almost never prunes and the per-tile consumer barrier costs 40% (H: 147 -> 206 ms); on tie-heavy
+// data (C5) it removes 92% of the chunk tests at equal time.  SKYCUBE_K3_SUPER=1 enables it (A/B runs).
+inline int super_enabled() {
+    const char *e = getenv("SKYCUBE_K3_SUPER");
+    return e && e[0] == '1';
+}
+
+template <int D, int MODE>
 void launch_c_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using G = Geo<D>;
-    using C = GeoC<D, TIES>;
+    using C = GeoC<D, MODE>;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
     const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
-    const size_t smem = sizeof(uint32_t) * (4 * kCStages + (size_t)kCStages * kCWarps * 33 * G::CW +
-                                            (size_t)tpc * (((G::CW + 3) & ~3) + (G::CW | 1)) + (size_t)tpc * C::PER +
-                                            kCWarps * 64);
-    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_c_kernel<D, TIES>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const size_t smem = sizeof(uint32_t) * (4 * kCStages + (size_t)kCStages * C::TW +
+                                            (size_t)tpc * (((G::CW + 3) & ~3) + (G::CW | 1)) + (size_t)tpc * C::PS +
+                                            (size_t)tpc + 2 * (size_t)ceil_div(tpc, 32) + kCWarps * 64);
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_c_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
-    k3_mdmc_c_kernel<D, TIES><<<blocks, (kCWarps + 1) * 32, smem, st>>>(
+    k3_mdmc_c_kernel<D, MODE><<<blocks, (kCWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc, rows32, c.tie.as<uint32_t>(), ext_rows32,
+        c.minord.as<uint32_t>(), c.supers_ext.as<uint32_t>(), super_enabled(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc, rows32, c.tie.as<uint32_t>(), ext_rows32,
         c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
 
+// Tie-heavy inputs (every dimension discrete enough for injective codes) or small d: the tie-exact state
+// (kModeDims, d <= 12) unless B_{p notin S+} itself is requested (ext rows), then kModeSmemTie.  Continuous
+// data at d > 10: ties are rare and go to a global row (kModeGlobalTie).
 template <int D>
 void launch_c(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     const bool all_exact = c.exact_mask == ((1u << D) - 1u);
-    if (D <= 10 || all_exact) launch_c_t<D, true>(c, j_begin, j_end, rows32, ext_rows32, st);
-    else launch_c_t<D, false>(c, j_begin, j_end, rows32, ext_rows32, st);
+    const char *m = getenv("SKYCUBE_K3_MODE");  // test hook: force a state mode
+    int mode = (D <= 10 || all_exact) ? (D <= 12 && !ext_rows32 ? kModeDims : kModeSmemTie) : kModeGlobalTie;
+    if (m && *m) {
+        mode = m[0] - '0';
+        if (mode == kModeDims && (D > 12 || ext_rows32)) mode = kModeSmemTie;
+    }
+    if (mode == kModeDims) {
+        if constexpr (D <= 12) launch_c_t<D, kModeDims>(c, j_begin, j_end, rows32, ext_rows32, st);
+    } else if (mode == kModeSmemTie) {
+        launch_c_t<D, kModeSmemTie>(c, j_begin, j_end, rows32, ext_rows32, st);
+    } else {
+        launch_c_t<D, kModeGlobalTie>(c, j_begin, j_end, rows32, ext_rows32, st);
+    }
 }
 
 template <int D, bool TIES>

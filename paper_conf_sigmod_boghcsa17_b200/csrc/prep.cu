@@ -85,6 +85,29 @@ __global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t 
     }
 }
 
+// Super-chunk corners: per tile of kTileChunks chunk records, the per-dimension minimum of the chunk
+// corners (the lower corner of 512 consecutive static-tree points).  One warp per tile.
+__global__ void build_supers_kernel(const uint32_t *__restrict__ chunks, int64_t ntiles, int cw, int cws,
+                                    uint32_t *__restrict__ supers) {
+    const int64_t t = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (t >= ntiles) return;
+    for (int k = 0; k < cws; k++) {
+        uint32_t lo = 0x7fffu, hi = 0x7fffu;
+        if (k < cw && lane < kTileChunks) {
+            const uint32_t w = chunks[((t * kTileChunks + lane) * 33 + 32) * (int64_t)cw + k];
+            lo = w & 0xffffu;
+            hi = w >> 16;
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+            hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+        }
+        if (lane == 0) supers[t * cws + k] = lo | (hi << 16);
+    }
+}
+
 // flags[t] = 1 iff t starts a run of equal (dim, key) in the per-dimension sorted order.
 __global__ void k2_flags_kernel(const uint64_t *__restrict__ comp_keys, int64_t n, int64_t total,
                                 uint32_t *__restrict__ flags) {
@@ -93,13 +116,15 @@ __global__ void k2_flags_kernel(const uint64_t *__restrict__ comp_keys, int64_t 
     flags[t] = (t % n == 0 || comp_keys[t] != comp_keys[t - 1]) ? 1u : 0u;
 }
 
-// R[dim] = number of distinct values of dimension dim.
+// R[dim] = number of distinct values of dimension dim; minord[dim] = key of its minimum value.
 __global__ void k2_distinct_kernel(const uint32_t *__restrict__ ex, const uint32_t *__restrict__ flags,
-                                   int64_t n, int d, uint32_t *__restrict__ R) {
+                                   const uint64_t *__restrict__ comp_keys, int64_t n, int d, uint32_t *__restrict__ R,
+                                   uint32_t *__restrict__ minord) {
     const int i = threadIdx.x;
     if (i >= d) return;
     const int64_t a = (int64_t)i * n, b = (int64_t)(i + 1) * n - 1;
     R[i] = (ex[b] + flags[b]) - (ex[a] + flags[a]) + 1u;
+    minord[i] = (uint32_t)comp_keys[a];
 }
 
 // code = dense rank if the dimension has <= 2^15 distinct values, else floor(rank * 2^15 / R):
@@ -240,6 +265,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.flags.ensure(sizeof(uint32_t) * nd);
     c.scanned.ensure(sizeof(uint32_t) * nd);
     c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
+    c.minord.ensure(sizeof(uint32_t) * kMaxD);
     c.nanflag.ensure(sizeof(uint32_t));
     c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
     c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
@@ -263,7 +289,8 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.L.count++;
     SKY_LAUNCH_CHECK();
     exclusive_scan_u32(c.flags.as<uint32_t>(), c.scanned.as<uint32_t>(), nd, c.scan_tmp.p, st, c.L);
-    k2_distinct_kernel<<<1, 32, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(), n, d, c.rbuf.as<uint32_t>());
+    k2_distinct_kernel<<<1, 32, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(), c.comp_keys.as<uint64_t>(), n,
+                                         d, c.rbuf.as<uint32_t>(), c.minord.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     k2_codes_kernel<<<blocks_for(nd, 256), 256, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(),
@@ -297,6 +324,12 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.L.count++;
     SKY_LAUNCH_CHECK();
     c.nchunks_all = nch;
+    const int64_t ntiles = ceil_div(nch, kTileChunks);
+    c.supers_all.ensure(sizeof(uint32_t) * ntiles * super_words(cw));
+    build_supers_kernel<<<blocks_for(ntiles * 32, 256), 256, 0, st>>>(c.chunks_all.as<uint32_t>(), ntiles, cw,
+                                                                      super_words(cw), c.supers_all.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
     SKY_CUDA(cudaStreamSynchronize(st));
     c.exact_mask = 0;
     for (int i = 0; i < d; i++)
@@ -380,6 +413,12 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.L.count++;
     SKY_LAUNCH_CHECK();
     c.nchunks_ext = nch;
+    const int64_t ntiles = ceil_div(nch, kTileChunks);
+    c.supers_ext.ensure(sizeof(uint32_t) * ntiles * super_words(cw));
+    build_supers_kernel<<<blocks_for(ntiles * 32, 256), 256, 0, st>>>(c.chunks_ext.as<uint32_t>(), ntiles, cw,
+                                                                      super_words(cw), c.supers_ext.as<uint32_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
     c.ext_ready = true;
 }
 

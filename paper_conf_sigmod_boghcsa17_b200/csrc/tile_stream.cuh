@@ -113,8 +113,23 @@ struct TileRing {
         mbar_arrive_expect_tx(&full[s], bytes);
         bulk_g2s(buf + (uint32_t)s * tile_words, src_tiles + t * (int64_t)tile_words, bytes, &full[s]);
     }
+    // Two-segment tile: words [0, na) from a + t*na, then words [na, na+nb) from b + t*nb (tile_words = na+nb).
+    __device__ __forceinline__ void issue2(const uint32_t *a, uint32_t na, const uint32_t *b, uint32_t nb,
+                                           int64_t t) const {
+        const int s = (int)(t % S);
+        if (t >= S) mbar_wait_sleep(&empty[s], (uint32_t)(((t / S) - 1) & 1));
+        mbar_arrive_expect_tx(&full[s], (na + nb) * 4u);
+        uint32_t *dst = buf + (uint32_t)s * tile_words;
+        bulk_g2s(dst, a + t * (int64_t)na, na * 4u, &full[s]);
+        bulk_g2s(dst + na, b + t * (int64_t)nb, nb * 4u, &full[s]);
+    }
     __device__ __forceinline__ void wait(int64_t t) const { mbar_wait(&full[t % S], (uint32_t)((t / S) & 1)); }
     __device__ __forceinline__ void release(int64_t t) const { mbar_arrive(&empty[t % S]); }
 };
+
+// Named barrier 1 over the consumer warps (the producer warp has left the CTA-wide barrier 0).
+__device__ __forceinline__ void consumer_sync(int nthreads) {
+    asm volatile("bar.sync 1, %0;" ::"r"(nthreads) : "memory");
+}
 
 }  // namespace sky

@@ -44,6 +44,11 @@ def check_against_oracle(x, res, ext=True):
     off, ids = oracle.lattice(want_rows, d)
     assert np.array_equal(res["offsets"], off)
     assert np.array_equal(res["ids"], ids)
+    # the product call (no B_{p in S+} rows requested) runs the tie-exact state for tie-heavy / low-d inputs
+    plain = sky.skycube_build(x)
+    bad = np.nonzero((plain["rows"] != want_rows).any(axis=1))[0]
+    assert bad.size == 0, f"{bad.size} rows differ without ext rows, first {bad[:5]}"
+    assert np.array_equal(plain["offsets"], off) and np.array_equal(plain["ids"], ids)
 
 
 def test_flights_table1():
@@ -162,3 +167,25 @@ def test_row_permutation_invariance():
     a = gpu(x)["rows"]
     b = gpu(x[perm])["rows"]
     assert np.array_equal(a[perm], b)
+
+
+@pytest.mark.parametrize("mode", ["0", "1", "2"])
+@pytest.mark.parametrize("d", [3, 6, 9, 11, 12])
+def test_k3_state_modes_tie_heavy(monkeypatch, mode, d):
+    """Every K3 state mode (global tie row / shared-memory tie row / per-dimension sets) on tie-heavy data,
+    including values tied at each dimension's minimum (Z_p of the per-dimension mode)."""
+    monkeypatch.setenv("SKYCUBE_K3_MODE", mode)
+    x = datagen.small_int_grid(700, d, 4, 300 + d)
+    x[::7, d - 1] = x[:, d - 1].min()
+    want = oracle.rows_b(x)
+    r = sky.skycube_build(x)
+    assert np.array_equal(r["rows"], want)
+    off, ids = oracle.lattice(want, d)
+    assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)
+
+
+def test_ct_like_tie_exact_state():
+    x = datagen.generate("ct", 6000, 10, 12)
+    want = oracle.rows_b(x)
+    r = sky.skycube_build(x)
+    assert np.array_equal(r["rows"], want)
