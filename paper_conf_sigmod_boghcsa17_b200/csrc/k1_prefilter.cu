@@ -23,7 +23,7 @@ namespace sky {
 namespace {
 
 constexpr int kWarps = kTileChunks;  // consumer warps = chunks per tile
-constexpr int kTasks = 2048;       // tasks per CTA
+constexpr int kTasks = 2048;       // tasks per CTA (<= 64 groups of 32)
 constexpr int kStages = 3;
 
 template <int CW>
@@ -113,7 +113,16 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k1_prefilter_kernel(
         const int64_t c = tile * kTileChunks + warp;
         if (c >= nchunks) continue;
         const int64_t qpos = c * 32 + lane;
-        for (int g = 0; g < ngroups; g++) {
+        // groups with work: lane l looks at groups l and l + 32 (ngroups <= kTasks / 32 = 64)
+        uint64_t gm;
+        {
+            const uint32_t n0 = lane < ngroups ? need[lane] & ~domw[lane] : 0u;
+            const uint32_t n1 = lane + 32 < ngroups ? need[lane + 32] & ~domw[lane + 32] : 0u;
+            gm = (uint64_t)__ballot_sync(0xffffffffu, n0 != 0) | ((uint64_t)__ballot_sync(0xffffffffu, n1 != 0) << 32);
+        }
+        while (gm) {
+            const int g = __ffsll((long long)gm) - 1;
+            gm &= gm - 1;
             const uint32_t nw = need[g] & ~domw[g];
             if (nw == 0) continue;
             const int tt = g * 32 + lane;

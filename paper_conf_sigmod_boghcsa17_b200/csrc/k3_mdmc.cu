@@ -405,7 +405,7 @@ struct GeoC {
     static constexpr int ROW = PS + ((Geo<D>::CW + 3) & ~3) + (Geo<D>::CW | 1);  // words per task
     static constexpr int TW = kCWarps * 33 * Geo<D>::CW + ((Geo<D>::CW + 3) & ~3);  // tile: 16 chunks + super corner
     static constexpr int RING = 4 * kCStages + kCStages * TW;  // words
-    static constexpr int NT0 = (kCSmemBytes / 4 - RING - 128 - kCWarps * 64) / (ROW + 1 + 1);
+    static constexpr int NT0 = (kCSmemBytes / 4 - RING - 128 - kCWarps * 128) / (ROW + 1 + 1);
     static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                         // tasks per CTA
 };
 
@@ -560,7 +560,8 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
     uint32_t *zm = state + tpc * C::PS;                             // [tpc] Z_p (kModeDims)
     const int TG = (tpc + 31) >> 5;
     uint32_t *needw = zm + tpc;                                      // [2][TG] tasks below the tile corner
-    uint32_t *mq = needw + 2 * TG + warp * 64;                       // per-warp miss queue [32][2]
+    uint32_t *mq = needw + 2 * TG + warp * 128;                      // per-warp miss queue [32][2]
+    uint32_t *wq = mq + 64;                                          // per-warp pair-test task queue [36]
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, kCWarps);
@@ -634,30 +635,9 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
         const int64_t c = tile * kCWarps + warp;
         if (c >= nchunks) continue;
         const int64_t qpos = c * 32 + lane;
-        for (int g = 0; g < ngroups; g++) {
-            const uint32_t nw = use_super ? need[g] : 0xffffffffu;
-            if (nw == 0) continue;
-            const int tt = min(g * 32 + lane, nt - 1);
-            uint32_t le[G::CW];
-#pragma unroll
-            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
-            const uint32_t Mb = gather_mask<G::NG>(le);
-            const uint32_t wb = state[tt * C::PS + (Mb >> 5)];
-            const bool needp = ((nw >> lane) & 1u) && g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
-            uint32_t todo = __ballot_sync(0xffffffffu, needp);
-            n_box += use_super ? __popc(nw) : min(32, nt - g * 32);
-            n_pair += 32u * __popc(todo);
-            while (todo) {
-                int ts[kCU];
-                int cnt = 0;
-#pragma unroll
-                for (int u = 0; u < kCU; u++) {
-                    ts[u] = g * 32 + (todo ? __ffs(todo) - 1 : 0);
-                    if (todo) {
-                        todo &= todo - 1;
-                        cnt++;
-                    }
-                }
+        // Pair tests are pooled across task groups in a per-warp queue and run kCU tasks at a time (independent
+        // chains), so that a batch is only partial once per chunk.
+        auto run_batch = [&](const int *ts, int cnt) {
                 uint32_t M[kCU], wd[kCU];
 #pragma unroll
                 for (int u = 0; u < kCU; u++) {
@@ -671,7 +651,7 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
                 uint32_t hit = 0xffffffffu;
 #pragma unroll
                 for (int u = 0; u < kCU; u++) hit &= __funnelshift_r(wd[u], wd[u], M[u]);
-                if (hit & 1u) continue;
+                if (hit & 1u) return;
 #pragma unroll
                 for (int u = 0; u < kCU; u++) {
                     if (u >= cnt) break;
@@ -719,8 +699,43 @@ __global__ void __launch_bounds__((kCWarps + 1) * 32, 1) k3_mdmc_c_kernel(
                     __syncwarp();
 #endif
                 }
+        };
+        int qn = 0;
+        uint32_t npair32 = 0;
+        for (int g = 0; g < ngroups; g++) {
+            const uint32_t nw = use_super ? need[g] : 0xffffffffu;
+            if (nw == 0) continue;
+            const int tt = min(g * 32 + lane, nt - 1);
+            uint32_t le[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
+            const uint32_t Mb = gather_mask<G::NG>(le);
+            const uint32_t wb = state[tt * C::PS + (Mb >> 5)];
+            const bool needp = ((nw >> lane) & 1u) && g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
+            const uint32_t todo = __ballot_sync(0xffffffffu, needp);
+            if (use_super) n_box += __popc(nw);
+            if (todo == 0) continue;
+            npair32 += __popc(todo);
+            if (needp) wq[qn + __popc(todo & ((1u << lane) - 1u))] = g * 32 + lane;
+            qn += __popc(todo);
+            __syncwarp();
+            while (qn >= kCU) {
+                qn -= kCU;
+                int ts[kCU];
+#pragma unroll
+                for (int u = 0; u < kCU; u++) ts[u] = wq[qn + u];
+                run_batch(ts, kCU);
             }
+            __syncwarp();
         }
+        if (qn > 0) {
+            int ts[kCU];
+#pragma unroll
+            for (int u = 0; u < kCU; u++) ts[u] = wq[min(u, qn - 1)];
+            run_batch(ts, qn);
+        }
+        if (!use_super) n_box += nt;
+        n_pair += 32ull * npair32;
     }
     if (counters) {
         if (lane == 0) {
@@ -777,7 +792,7 @@ void launch_c_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32
     const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
     const size_t smem = sizeof(uint32_t) * (4 * kCStages + (size_t)kCStages * C::TW +
                                             (size_t)tpc * (((G::CW + 3) & ~3) + (G::CW | 1)) + (size_t)tpc * C::PS +
-                                            (size_t)tpc + 2 * (size_t)ceil_div(tpc, 32) + kCWarps * 64);
+                                            (size_t)tpc + 2 * (size_t)ceil_div(tpc, 32) + kCWarps * 128);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_c_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_mdmc_c_kernel<D, MODE><<<blocks, (kCWarps + 1) * 32, smem, st>>>(
