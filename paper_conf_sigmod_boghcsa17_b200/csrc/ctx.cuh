@@ -88,7 +88,6 @@ void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cu
 void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
                      cudaStream_t st);
 
-constexpr int kPrefilterTile = 256;  // sorted positions per K1 block
 constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
 constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole
 constexpr int kTileChunks = 16;         // chunks per competitor tile (one super-chunk of 512 points)

@@ -4,7 +4,7 @@ Sharding (the paper's device-level data parallelism of MDMC, L
 task is independent, there is no need for synchronisation"):
 
   1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic)
-  2. K1 prefilter                                 blocks of 2048 prepared (static-tree order) positions,
+  2. K1 prefilter                                 blocks of 512 static-tree positions,
                                                   block b on rank b % world
   3. exchange S+ flags                            all_reduce(MAX) of a uint8 flag vector (NCCL over NVLink)
   4. install S+ (replicated)
@@ -26,7 +26,7 @@ import torch.distributed as dist
 
 from . import Context, words_per_row
 
-PREFILTER_BLOCK = 2048  # prepared positions per K1 CTA (k1_prefilter.cu kTasks)
+PREFILTER_BLOCK = 512  # tree positions per K1 CTA (k1_prefilter.cu kTasks)
 GROUP = 32
 
 
