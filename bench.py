@@ -263,7 +263,7 @@ def run_ours(args):
     # roofline of the dominant kernel (K3 MDMC), duration from CUDA events on its stream; its work is
     # the tests it must run after static-tree pruning (device counters), not the n_ext^2 pairs it resolves
     mdmc_ms = phase["mdmc"]
-    tests = work["k3_box"] + work["k3_pair"]
+    tests = work["k3_box"] + work.get("k3_sub", 0) + work["k3_pair"]
     ops = tests * algorithmic_ops_per_test(d)
     achieved = ops / (mdmc_ms / 1e3) / 1e12
     peak = alu_peak_ops(sm_mhz) / 1e12
@@ -275,7 +275,7 @@ def run_ours(args):
                    "l2": "256 MB buffer written between timed steps",
                    "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
         "phases_ms": phase,
-        "work_per_step": {**work, "pairs_resolved_by_chunk_tests": 32 * work["k3_box"] - work["k3_pair"]},
+        "work_per_step": work,
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
                      "frac": achieved / peak, "traffic": None,
@@ -305,15 +305,18 @@ def measure_e2e(args, x, eng, world, rank, dev, pairs):
         r = sky.skycube_build_raw(x, stats=True)  # warm (pinned pools, contexts)
         d2h = 4 * r.n_ext + 4 * n * sky.words_per_row(d) + 8 * ((1 << d) + 1) + 4 * int(r.offsets()[-1])
         r.close()
-        times = []
+        times, phases = [], []
         for _ in range(args.e2e_steps):
             t0 = time.perf_counter()
-            r = sky.skycube_build_raw(x)
+            r = sky.skycube_build_raw(x, stats=True)
             times.append(time.perf_counter() - t0)
+            phases.append(r.stats)
             r.close()
         t = statistics.median(times)
+        keys = ("ms_h2d", "ms_sort", "ms_prefilter", "ms_mdmc", "ms_compact", "ms_d2h", "ms_total")
         return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
-                "ms_per_step": t * 1e3, "api": "skycube_build_ex (C-ABI, host buffers, pinned result pool)"}
+                "ms_per_step": t * 1e3, "api": "skycube_build_ex (C-ABI, host buffers, pinned result pool)",
+                "phases_ms": {k: statistics.median(p[k] for p in phases) for k in keys}}
     # N > 1: pinned host input -> every rank H2D -> sharded pipeline -> rank 0 D2H of all outputs
     host = torch.from_numpy(x).pin_memory()
     times = []

@@ -260,7 +260,7 @@ class Context:
         a = np.zeros(8, np.int64)
         _check(lib().skycube_ctx_counters(self._h, a.ctypes.data_as(ctypes.c_void_p)))
         return {"k1_box": int(a[0]), "k1_pair": int(a[1]), "k3_box": int(a[2]), "k3_pair": int(a[3]),
-                "k3_miss": int(a[4])}
+                "k3_miss": int(a[4]), "k3_sub": int(a[5])}
 
     def info(self):
         m, W, ex = ctypes.c_int64(), ctypes.c_uint32(), ctypes.c_uint32()

@@ -296,7 +296,7 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
                            &c.counts, &c.scan_tmp, &c.flags, &c.scanned, &c.rbuf, &c.minord, &c.nanflag, &c.codes_id,
                            &c.codes_sorted, &c.ord_sorted, &c.ext_id_flag, &c.ext_idx, &c.key_flag, &c.key_idx,
                            &c.ext_ids, &c.p_codes, &c.p_ord, &c.q_codes, &c.q_ord, &c.tie, &c.lat_counts,
-                           &c.scan64_tmp, &c.chunks_all, &c.chunks_ext, &c.supers_all, &c.supers_ext, &c.counters, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
+                           &c.scan64_tmp, &c.chunks_all, &c.chunks_ext, &c.supers_all, &c.counters, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
                            &ctx->membership, &ctx->offsets, &ctx->ids})
         b->release();
     delete ctx;

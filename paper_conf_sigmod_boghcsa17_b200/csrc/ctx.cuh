@@ -66,10 +66,10 @@ struct Ctx {
     DevBuf q_codes;     // u16 [mpad*dp]  S+ in static-tree order (MDMC competitor stream)
     DevBuf q_ord;       // u32 [m*d]
     DevBuf tie;         // u32 tiled rows: tie contributions to B_{p notin S}
-    DevBuf chunks_all;  // u32 [n/32][33][cw]  chunk records of all points (K1 competitors)
-    DevBuf chunks_ext;  // u32 [m/32][33][cw]  chunk records of S+ (K3 competitors)
+    DevBuf chunks_all;  // u32 [n/32][kRecAll][cw]  chunk records of all points (K1 competitors)
+    DevBuf chunks_ext;  // u32 [m/32][kRecExt][cw]  chunk records of S+ with sub-chunk corners (K3 competitors)
     DevBuf chunk_keys, chunk_perm, q_codes_alt, q_ord_alt;  // chunk visiting order (strongest corner first)
-    DevBuf supers_all, supers_ext;  // u32 [tiles][super_words(cw)]  lower corner of each tile of 16 chunks
+    DevBuf supers_all;  // u32 [tiles][super_words(cw)]  lower corner of each tile of 16 chunks (K1)
     int64_t nchunks_all = 0, nchunks_ext = 0;
     DevBuf lat_counts;  // u64 [2^d * nchunks]
     DevBuf counters;    // u64 [8]: K1 box tests, K1 pair tests, K3 box tests, K3 pair tests, K3 misses
@@ -91,6 +91,9 @@ void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *
 constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
 constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole
 constexpr int kTileChunks = 16;         // chunks per competitor tile (one super-chunk of 512 points)
+constexpr int kSubSize = 4;             // points per sub-chunk (K3 level below the chunk)
+constexpr int kRecAll = 33;             // K1 chunk record rows: 32 points + corner
+constexpr int kRecExt = 33 + 32 / kSubSize;  // K3 chunk record rows: + 8 sub-chunk corners
 inline int super_words(int cw) { return (cw + 3) & ~3; }  // super-corner record words (16-byte multiple)
 
 }  // namespace sky

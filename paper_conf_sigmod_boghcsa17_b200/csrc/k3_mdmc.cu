@@ -18,8 +18,11 @@
 //   box pass   lane l tests task 32g+l against the chunk corner (SWAR over 16-bit code lanes with guard
 //              bits, gathered to a d-bit mask with a byte permute and a carry-free multiply per 4
 //              dimensions) and probes the task's state; a ballot gives the tasks whose chunk must be opened;
-//   pair pass  queued tasks, kCU at a time (independent chains): every lane forms M = B_{code(q)<=code(p)}
-//              (a superset of L: codes are monotone, Λ3) and probes bit M; set => skip (Λ4);
+//   sub pass   opened tasks, 4 at a time: lane (u, s) tests task u against the corner of sub-chunk s (4
+//              points, the level below); opened (task, sub-chunk) items are queued;
+//   pair pass  8 items at a time: lane (k, r) takes member r of item k's sub-chunk (shuffled from the lane
+//              that holds it) and forms M = B_{code(q)<=code(p)} (a superset of L: codes are monotone, Λ3),
+//              then probes bit M; set => skip (Λ4);
 //   miss       (rare: ~0.3% of pair tests on the anticorrelated headline) the lane computes the exact L, S
 //              (strict SWAR compare plus exact keys on tied, non-injective codes); then the whole warp
 //              expands each contributing competitor word-parallel (Alg. 3 line 12: for the word index w, the
@@ -61,7 +64,6 @@ struct Geo {
 constexpr int kWarps = 16;                // consumer warps = chunks per tile (+1 producer warp)
 constexpr int kStages = 4;                // TMA ring depth
 constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
-constexpr int kCU = 4;                    // tasks per pair-pass batch
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");
 
@@ -71,10 +73,10 @@ struct GeoK3 {
     static constexpr int PS = PER | 1;                                   // odd task stride (bank spread)
     static constexpr int CWP = Geo<D>::CW | 1;                           // odd code stride (box pass)
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
-    static constexpr int REC = 33 * Geo<D>::CW;                          // chunk record words
+    static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
     static constexpr int TW = kWarps * REC;                              // tile words
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
-    static constexpr int QW = 64;                                        // per-warp queue words
+    static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
     static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
     static constexpr int NT0 = (kSmemBytes / 4 - RING - kWarps * QW - 64) / ROW;
     static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                   // tasks per CTA
@@ -242,7 +244,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     uint32_t *state = pH + tpc * CWP;          // [tpc][PS]
     uint32_t *zm = state + tpc * C::PS;        // [tpc] Z_p (kModeDims)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    uint32_t *wq = zm + tpc + warp * C::QW;    // per-warp pair-test task queue (<= kCU - 1 + 32 entries)
+    uint32_t *wq = zm + tpc + warp * C::QW;    // per-warp queue of opened tasks (<= 3 + 32 entries)
+    uint32_t *iq = wq + 40;                    // per-warp queue of opened (task, sub-chunk) items (<= 7 + 32)
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
@@ -281,67 +284,95 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         return;
     }
     const int ngroups = (nt + 31) >> 5;
-    unsigned long long n_box = 0, n_pair = 0, n_miss = 0;
+    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t *rec = ring.stage(tile) + warp * REC;
-        uint32_t q[G::CW], mn[G::CW];
+        // this lane's competitor, the chunk corner, and the corner of sub-chunk (lane & 7) — the level below
+        // the chunk in the static tree (4 points) — all read before the stage is released
+        uint32_t q[G::CW], mn[G::CW], sc[G::CW];
 #pragma unroll
         for (int k = 0; k < G::CW; k++) {
             q[k] = rec[lane * G::CW + k];
             mn[k] = rec[32 * G::CW + k];
+            sc[k] = rec[(33 + (lane & 7)) * G::CW + k];
         }
+        // The loads above are still in flight (their values are first used much later): complete them before
+        // the stage is handed back to the TMA producer, or the next tile's bulk copy can overwrite the stage
+        // under them (observed as rare missing dominations at d >= 13 without this fence).
+        __threadfence_block();
         __syncwarp();
         if (lane == 0) ring.release(tile);
         const int64_t c = tile * kWarps + warp;
         if (c >= nchunks) continue;
         const int64_t qpos = c * 32 + lane;
 
-        // kCU queued tasks against the lane's competitor (independent chains), then misses (Alg. 3 10-12)
-        auto run_batch = [&](const int *ts, int cnt) {
-            uint32_t M[kCU], wd[kCU];
+        // pair pass over packed items (task t, sub-chunk s): lane (k, r) = item k, member r of sub-chunk s; the
+        // competitor comes from the lane that holds it (shuffle); misses run Alg. 3 lines 10-12 cooperatively
+        auto pair_pass = [&](int base, int cnt) {
+            const int k8 = lane >> 2, r = lane & 3;
+            const uint32_t it = iq[base + min(k8, cnt - 1)];
+            const int t = (int)(it >> 3), src = (int)((it & 7u) << 2) + r;
+            uint32_t qq[G::CW], x[G::CW];
 #pragma unroll
-            for (int u = 0; u < kCU; u++) {
-                uint32_t x[G::CW];
-                load_row<G::CW>(pV + ts[u] * CWV, x);
+            for (int k = 0; k < G::CW; k++) qq[k] = __shfl_sync(0xffffffffu, q[k], src);
+            load_row<G::CW>(pV + t * CWV, x);
 #pragma unroll
-                for (int k = 0; k < G::CW; k++) x[k] -= q[k];  // guard <=> code(q) <= code(p)
-                M[u] = gather_mask<G::NG>(x);
-                wd[u] = state[ts[u] * C::PS + (M[u] >> 5)];
+            for (int k = 0; k < G::CW; k++) x[k] -= qq[k];  // guard <=> code(q) <= code(p)
+            const uint32_t M = gather_mask<G::NG>(x);
+            const uint32_t wd = state[t * C::PS + (M >> 5)];
+            const bool miss = k8 < cnt && !(__funnelshift_r(wd, wd, M) & 1u);
+            if (!__any_sync(0xffffffffu, miss)) return;  // Λ4 for every lane
+            uint32_t L = 0, S = 0;
+            if (miss) {
+                n_miss++;
+                exact_masks<D>(pH + t * CWP, qq, M, inexact, q_ord + (c * 32 + src) * D, p_ord + (j0 + t) * D, L, S);
+                const uint32_t *st = state + t * C::PS;
+                if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
             }
-            uint32_t hit = 0xffffffffu;
-#pragma unroll
-            for (int u = 0; u < kCU; u++) hit &= __funnelshift_r(wd[u], wd[u], M[u]);  // bit M of the probe set
-            if (__all_sync(0xffffffffu, hit & 1u)) return;  // Λ4 for every lane and task of the batch
-#pragma unroll
-            for (int u = 0; u < kCU; u++) {
-                if (u >= cnt) break;
-                const int t = ts[u];
-                uint32_t *st = state + t * C::PS;
-                uint32_t L = 0, S = 0;
-                if (!(__funnelshift_r(wd[u], wd[u], M[u]) & 1u)) {
-                    n_miss++;
-                    exact_masks<D>(pH + t * CWP, q, M[u], inexact, q_ord + qpos * D, p_ord + (j0 + t) * D, L, S);
-                    if (S != 0 && L != M[u] && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
-                }
-                uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
-                if (!todo) continue;
-                const int64_t jt = j0 + t;
+            uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
+            while (todo) {
+                const int from = __ffs(todo) - 1;
+                todo &= todo - 1;
+                const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
+                const int tb = __shfl_sync(0xffffffffu, t, from);
+                uint32_t *st = state + tb * C::PS;
+                const int64_t jt = j0 + tb;
                 uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-                const uint32_t z = MODE == kModeDims ? zm[t] : 0u;
-                while (todo) {
-                    const int src = __ffs(todo) - 1;
-                    todo &= todo - 1;
-                    const uint32_t Sb = __shfl_sync(0xffffffffu, S, src), Lb = __shfl_sync(0xffffffffu, L, src);
-                    expand<D, MODE>(st, tr, TIES ? 1 : 32, Lb, Sb, z, lane);
-                }
+                expand<D, MODE>(st, tr, TIES ? 1 : 32, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
             }
         };
 
-        // box pass; the tasks whose chunk must be opened are pooled across task groups in a per-warp queue,
-        // so that a batch is only partial once per chunk
+        // sub-chunk pass: lane (u, s) tests queued task u against sub-chunk corner s; the opened (task,
+        // sub-chunk) items are queued and run 8 per pair pass
+        int iqn = 0;
+        uint32_t nsub32 = 0, nitem32 = 0;
+        auto sub_pass = [&](int base, int cnt) {
+            const int u = lane >> 3;
+            const int t = wq[base + min(u, cnt - 1)];
+            uint32_t x[G::CW];
+            load_row<G::CW>(pV + t * CWV, x);
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) x[k] -= sc[k];  // guard <=> sub-corner <= p
+            const uint32_t Ms = gather_mask<G::NG>(x);
+            const uint32_t ws = state[t * C::PS + (Ms >> 5)];
+            const bool open = u < cnt && !(__funnelshift_r(ws, ws, Ms) & 1u);
+            const uint32_t ob = __ballot_sync(0xffffffffu, open);
+            nsub32 += 8 * cnt;
+            if (!ob) return;
+            nitem32 += __popc(ob);
+            if (open) iq[iqn + __popc(ob & ((1u << lane) - 1u))] = ((uint32_t)t << 3) | (uint32_t)(lane & 7);
+            iqn += __popc(ob);
+            __syncwarp();
+            while (iqn >= 8) {
+                iqn -= 8;
+                pair_pass(iqn, 8);
+            }
+            __syncwarp();
+        };
+
+        // box pass; the tasks whose chunk must be opened are pooled across task groups in a per-warp queue
         int qn = 0;
-        uint32_t npair32 = 0;
         for (int g = 0; g < ngroups; g++) {
             const int tt = min(g * 32 + lane, nt - 1);
             uint32_t le[G::CW];
@@ -352,27 +383,21 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             const bool open = g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
             const uint32_t todo = __ballot_sync(0xffffffffu, open);
             if (todo == 0) continue;
-            npair32 += __popc(todo);
             if (open) wq[qn + __popc(todo & ((1u << lane) - 1u))] = g * 32 + lane;
             qn += __popc(todo);
             __syncwarp();
-            while (qn >= kCU) {
-                qn -= kCU;
-                int ts[kCU];
-#pragma unroll
-                for (int u = 0; u < kCU; u++) ts[u] = wq[qn + u];
-                run_batch(ts, kCU);
+            while (qn >= 4) {
+                qn -= 4;
+                sub_pass(qn, 4);
             }
             __syncwarp();
         }
-        if (qn > 0) {
-            int ts[kCU];
-#pragma unroll
-            for (int u = 0; u < kCU; u++) ts[u] = wq[min(u, qn - 1)];
-            run_batch(ts, qn);
-        }
+        if (qn > 0) sub_pass(0, qn);
+        if (iqn > 0) pair_pass(0, iqn);
+        __syncwarp();
+        n_sub += nsub32;
+        n_pair += 4ull * nitem32;
         n_box += nt;
-        n_pair += 32ull * npair32;
     }
     if (counters) {
         if (lane == 0) {
@@ -380,7 +405,10 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             atomicAdd(&counters[3], n_pair);
         }
         for (int o = 16; o; o >>= 1) n_miss += __shfl_xor_sync(0xffffffffu, n_miss, o);
-        if (lane == 0) atomicAdd(&counters[4], n_miss);
+        if (lane == 0) {
+            atomicAdd(&counters[4], n_miss);
+            atomicAdd(&counters[5], n_sub);
+        }
     }
     consumer_sync(kWarps * 32);
     // B_{p notin S} -> membership row (its complement; bit 0, the empty subspace, is never a member)

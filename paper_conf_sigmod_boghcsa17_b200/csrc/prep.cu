@@ -64,22 +64,25 @@ __global__ void morton_kernel(const uint16_t *__restrict__ codes, const uint32_t
     perm[p] = (uint32_t)p;
 }
 
-// Chunk records: 32 consecutive points' code words, then the per-dimension minimum code words
-// (the chunk's lower corner).  One warp per chunk.
-__global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw,
+// Chunk records (rec_rows x cw words): 32 consecutive points' code words, then the per-dimension minimum
+// code words (the chunk's lower corner), then — when rec_rows == kRecExt — the lower corners of the 8
+// sub-chunks of 4 consecutive points (the level below, K3).  One warp per chunk.
+__global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw, int rec_rows,
                                     uint32_t *__restrict__ chunks) {
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (c >= nchunks) return;
-    uint32_t *rec = chunks + c * (int64_t)(33 * cw);
+    uint32_t *rec = chunks + c * (int64_t)(rec_rows * cw);
     for (int k = 0; k < cw; k++) {
         const uint32_t w = codes[(c * 32 + lane) * cw + k];
         rec[lane * cw + k] = w;
         uint32_t lo = w & 0xffffu, hi = w >> 16;
 #pragma unroll
-        for (int o = 16; o; o >>= 1) {
+        for (int o = 1; o < 32; o <<= 1) {
             lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
             hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+            if (o == kSubSize / 2 && rec_rows == kRecExt && (lane & (kSubSize - 1)) == 0)
+                rec[(33 + lane / kSubSize) * cw + k] = lo | (hi << 16);  // sub-chunk corner
         }
         if (lane == 0) rec[32 * cw + k] = lo | (hi << 16);
     }
@@ -95,7 +98,7 @@ __global__ void build_supers_kernel(const uint32_t *__restrict__ chunks, int64_t
     for (int k = 0; k < cws; k++) {
         uint32_t lo = 0x7fffu, hi = 0x7fffu;
         if (k < cw && lane < kTileChunks) {
-            const uint32_t w = chunks[((t * kTileChunks + lane) * 33 + 32) * (int64_t)cw + k];
+            const uint32_t w = chunks[((t * kTileChunks + lane) * kRecAll + 32) * (int64_t)cw + k];
             lo = w & 0xffffu;
             hi = w >> 16;
         }
@@ -202,7 +205,7 @@ __global__ void chunk_key_kernel(const uint32_t *__restrict__ chunks, int64_t nc
                                  uint64_t *__restrict__ keys, uint32_t *__restrict__ perm) {
     const int64_t ch = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (ch >= nch) return;
-    const uint32_t *mn = chunks + ch * (int64_t)(33 * cw) + 32 * cw;
+    const uint32_t *mn = chunks + ch * (int64_t)(kRecExt * cw) + 32 * cw;
     uint64_t s = 0;
     for (int i = 0; i < d; i++) s += (mn[i >> 1] >> (16 * (i & 1))) & 0xffffu;
     keys[ch] = s;
@@ -270,7 +273,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
     c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
     c.ord_sorted.ensure(sizeof(uint32_t) * nd);
-    c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * 33 * cw);
+    c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * kRecAll * cw);
 
     SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
     k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, c.ord.as<uint32_t>(), c.comp_keys.as<uint64_t>(),
@@ -319,7 +322,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     SKY_LAUNCH_CHECK();
     const int64_t nch = ceil_div(n, 32);
     pad_codes(c.codes_sorted.as<uint32_t>(), nch * 32, npad, cw, st, c.L);
-    build_chunks_kernel<<<blocks_for((npad / 32) * 32, 256), 256, 0, st>>>(c.codes_sorted.as<uint32_t>(), npad / 32, cw,
+    build_chunks_kernel<<<blocks_for((npad / 32) * 32, 256), 256, 0, st>>>(c.codes_sorted.as<uint32_t>(), npad / 32, cw, kRecAll,
                                                                           c.chunks_all.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
@@ -366,7 +369,7 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.p_ord.ensure(sizeof(uint32_t) * mm * d);
     c.q_codes.ensure(sizeof(uint16_t) * mpad * c.dp);
     c.q_ord.ensure(sizeof(uint32_t) * mpad * d);
-    c.chunks_ext.ensure(sizeof(uint32_t) * (mpad / 32) * 33 * cw);
+    c.chunks_ext.ensure(sizeof(uint32_t) * (mpad / 32) * kRecExt * cw);
     ext_build_id_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(),
                                                             c.codes_id.as<uint32_t>(), c.ord.as<uint32_t>(), n, d, cw,
                                                             c.ext_ids.as<int32_t>(), c.p_codes.as<uint32_t>(),
@@ -388,7 +391,7 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.chunk_perm.ensure(sizeof(uint32_t) * nch);
     c.q_codes_alt.ensure(sizeof(uint32_t) * mpad * cw);
     c.q_ord_alt.ensure(sizeof(uint32_t) * mpad * d);
-    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw,
+    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw, kRecExt,
                                                               c.chunks_ext.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
@@ -408,17 +411,11 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     std::swap(c.q_ord, c.q_ord_alt);
     pad_codes(c.q_codes.as<uint32_t>(), nch * 32, mpad, cw, st, c.L);
     pad_ord(c.q_ord.as<uint32_t>(), nch * 32, mpad, d, st, c.L);
-    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw,
+    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw, kRecExt,
                                                               c.chunks_ext.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     c.nchunks_ext = nch;
-    const int64_t ntiles = ceil_div(nch, kTileChunks);
-    c.supers_ext.ensure(sizeof(uint32_t) * ntiles * super_words(cw));
-    build_supers_kernel<<<blocks_for(ntiles * 32, 256), 256, 0, st>>>(c.chunks_ext.as<uint32_t>(), ntiles, cw,
-                                                                      super_words(cw), c.supers_ext.as<uint32_t>());
-    c.L.count++;
-    SKY_LAUNCH_CHECK();
     c.ext_ready = true;
 }
 

@@ -189,3 +189,14 @@ def test_ct_like_tie_exact_state():
     want = oracle.rows_b(x)
     r = sky.skycube_build(x)
     assert np.array_equal(r["rows"], want)
+
+
+@pytest.mark.parametrize("d", [13, 14])
+def test_repeat_builds_multi_tile_high_d(d):
+    """Several tiles of the competitor ring at d >= 13 (CW = 8), built repeatedly: a missing fence between the
+    last reads of a ring stage and its release once let the next bulk copy overwrite the stage under them
+    (rare missing dominations).  Every repetition must be bit-exact."""
+    x = datagen.generate("A", 2500, d, 6)
+    want = oracle.rows_b(x)
+    for _ in range(6):
+        assert np.array_equal(sky.skycube_build(x)["rows"], want)
