@@ -125,6 +125,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--clocks-log", default=None)
+    ap.add_argument("--output", default="lattice", choices=["lattice", "hashcube", "both"],
+                    help="skycube representation built by each step: the lattice (K4, Fig. 1a, default), the "
+                         "HashCube (K5, w=32, Alg. 3 line 13 / Fig. 1b) or both")
+    ap.add_argument("--max-level", type=int, default=0, help="partial skycube d' (Appendix A.2); 0 = full")
     return ap.parse_args()
 
 
@@ -207,8 +211,12 @@ def run_ours(args):
     eng = DeviceSkycube(local)
     names = ["t0", "t1", "t2", "t3", "t4"]
 
+    lists = args.output in ("lattice", "both")
+    hc_w = 32 if args.output in ("hashcube", "both") else 0
+
     def step(events=None):
-        return eng.build(pts, lists=True, membership=True, events=events)
+        return eng.build(pts, lists=lists, membership=True, events=events, hashcube_w=hc_w,
+                         max_level=args.max_level)
 
     out = None
     for _ in range(args.warmup):
@@ -217,7 +225,8 @@ def run_ours(args):
         out = step()
     torch.cuda.synchronize()
     m = out["n_ext"]
-    total_ids = out["total_ids"]
+    total_ids = out.get("total_ids", 0)
+    hc_ids = int(out["hashcube"]["ids"].numel()) if hc_w else None
     ev = [{k: torch.cuda.Event(enable_timing=True) for k in names} for _ in range(args.steps)]
     launches0 = eng.launches
     cnt0 = eng.ctx.counters()
@@ -272,6 +281,8 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": workload(cfg), "n": n, "d": d, "n_ext": m, "pairs": pairs, "total_ids": total_ids,
+                   "output": args.output + (f" (w=32, {hc_ids} stored ids)" if hc_w else ""),
+                   "max_level": args.max_level or d,
                    "l2": "256 MB buffer written between timed steps",
                    "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
         "phases_ms": phase,
@@ -302,20 +313,35 @@ def measure_e2e(args, x, eng, world, rank, dev, pairs):
     n, d = x.shape
     if world == 1:
         import paper_conf_sigmod_boghcsa17_b200 as sky
-        r = sky.skycube_build_raw(x, stats=True)  # warm (pinned pools, contexts)
-        d2h = 4 * r.n_ext + 4 * n * sky.words_per_row(d) + 8 * ((1 << d) + 1) + 4 * int(r.offsets()[-1])
+        if args.output == "hashcube":
+            def call():
+                return sky.skycube_build_hashcube_raw(x, 32, stats=True, max_level=args.max_level)
+
+            def d2h_bytes(r):
+                a = r.arrays()
+                return sum(int(v.nbytes) for v in a.values())
+            api = "skycube_build_hashcube (C-ABI, host buffers, pinned result pool)"
+        else:
+            def call():
+                return sky.skycube_build_raw(x, stats=True, lists=args.output != "hashcube", max_level=args.max_level)
+
+            def d2h_bytes(r):
+                return 4 * r.n_ext + 4 * n * sky.words_per_row(d) + 8 * ((1 << d) + 1) + 4 * int(r.offsets()[-1])
+            api = "skycube_build_ex (C-ABI, host buffers, pinned result pool)"
+        r = call()  # warm (pinned pools, contexts)
+        d2h = d2h_bytes(r)
         r.close()
         times, phases = [], []
         for _ in range(args.e2e_steps):
             t0 = time.perf_counter()
-            r = sky.skycube_build_raw(x, stats=True)
+            r = call()
             times.append(time.perf_counter() - t0)
             phases.append(r.stats)
             r.close()
         t = statistics.median(times)
         keys = ("ms_h2d", "ms_sort", "ms_prefilter", "ms_mdmc", "ms_compact", "ms_d2h", "ms_total")
         return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
-                "ms_per_step": t * 1e3, "api": "skycube_build_ex (C-ABI, host buffers, pinned result pool)",
+                "ms_per_step": t * 1e3, "api": api,
                 "phases_ms": {k: statistics.median(p[k] for p in phases) for k in keys}}
     # N > 1: pinned host input -> every rank H2D -> sharded pipeline -> rank 0 D2H of all outputs
     host = torch.from_numpy(x).pin_memory()

@@ -64,6 +64,11 @@ typedef struct {
     int32_t num_gpus;     /* reserved for the single-process multi-GPU path; 0 or 1 = one GPU */
     int32_t device;       /* CUDA device ordinal to use */
     uint32_t flags;       /* SKYCUBE_* flags */
+    int32_t max_level;    /* partial skycube (Appendix A.2): 0 = full skycube; d' in [1, d] =
+                             only the subspaces with |delta| <= d' are computed and reported -- membership
+                             bits of every delta with |delta| > d' are 0 and their lists are empty
+                             (reading P1: "no correctness guarantee is offered for the skyline
+                             of said delta", L1180) */
 } skycube_opts;
 
 typedef struct {
@@ -88,6 +93,49 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
 /* Release every buffer of `out` and zero it.  Idempotent; safe on a zeroed struct. */
 void skycube_free(skycube_result *out);
 
+/* ------------------------------------------------------------------------------------------------
+ * HashCube output (Alg. 3 lines 1 and 13, L320; Appendix B.1; Fig. 1b).
+ * Point p is represented by B_{p notin S}: 2^d - 1 bits, bit delta-1 set <=> p is dominated in delta
+ * (the shifted order of L79).  It is cut into n_words = ceil((2^d - 1) / w) words of w bits (word k =
+ * subspaces k*w+1 .. k*w+w; the last word may be shorter) and word k is hashed by h_k: key = the word's
+ * value, value = the ids of the points with that key.  A point whose word is all set (dominated in all
+ * of the word's subspaces) is not stored (L1278); points outside S+(P) are never stored.
+ * The hash maps are returned as sorted arrays (reading H1): the keys of word k are
+ * keys[word_offsets[k] .. word_offsets[k+1]) ascending, the ids of key u are
+ * ids[key_offsets[u] .. key_offsets[u+1]) ascending.
+ * Retrieval of S_delta (L1280, reading Q6): the lists of h_{(delta-1)/w} whose key has bit (delta-1) % w
+ * NOT set -- see skycube_hashcube_query.
+ * ------------------------------------------------------------------------------------------------ */
+typedef struct {
+    int32_t d;
+    uint32_t w;               /* word length, 1..32 (the paper's GPU HashCube uses 32, L158) */
+    int64_t n;                /* number of points */
+    int64_t n_ext;            /* |S+(P)| */
+    int64_t n_words;          /* ceil((2^d - 1) / w) hash functions */
+    int64_t total_keys;       /* distinct (word, key) pairs stored */
+    int64_t total_ids;        /* stored ids: at most n_ext * n_words */
+    int64_t *word_offsets;    /* [n_words + 1] */
+    uint32_t *keys;           /* [total_keys]  bit b <=> dominated in subspace k*w + b + 1 */
+    int64_t *key_offsets;     /* [total_keys + 1] */
+    int32_t *ids;             /* [total_ids] */
+} skycube_hashcube;
+
+/* Build the skycube of points[n*d] (as skycube_build) and return it as a HashCube with word length w.
+ * opts (nullable): device, max_level (partial skycube: subspaces above d' are reported as dominated,
+ * which the HashCube then compresses away); flags and num_gpus are ignored.  Buffers are pinned host
+ * memory owned by the library; release with skycube_hashcube_free.  Errors as skycube_build_ex, plus
+ * EINVAL for w outside [1, 32] and ENOMEM when n_ext * n_words >= 2^32. */
+skycube_status skycube_build_hashcube(const float *points, int64_t n, int32_t d, uint32_t w, const skycube_opts *opts,
+                                      skycube_hashcube *out, skycube_stats *stats);
+
+/* Release every buffer of `hc` and zero it.  Idempotent; safe on a zeroed struct. */
+void skycube_hashcube_free(skycube_hashcube *hc);
+
+/* Subspace skyline query on a HashCube (the read path, L1280): *count = |S_delta(P)|; if ids != NULL it
+ * must hold *count entries (call once with ids == NULL to size it) and receives the ids ascending.
+ * Host-side; EINVAL for delta outside [1, 2^d - 1] or a zeroed hc. */
+skycube_status skycube_hashcube_query(const skycube_hashcube *hc, uint32_t delta, int32_t *ids, int64_t *count);
+
 const char *skycube_strerror(skycube_status s);
 const char *skycube_last_error(void);   /* thread-local detail of the last error */
 
@@ -109,7 +157,7 @@ void skycube_ctx_destroy(skycube_ctx *ctx);
 skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, void *stream);
 
 /* Phase 2: extended-skyline prefilter (K1).  The prepared (static-tree) positions are cut into blocks of
- * 2048; this call processes the blocks b with b % tile_step == tile_offset (interleaving balances ranks).
+ * 512 (one K1 CTA each); this call processes the blocks b with b % tile_step == tile_offset (interleaving balances ranks).
  * Writes d_ext_sorted[s] = 1 iff the point at prepared position s is in S+(P), 0 otherwise, for the
  * positions of those blocks only.  d_ext_sorted: [n] uint8 device buffer owned by the caller. */
 skycube_status skycube_dev_prefilter(skycube_ctx *ctx, int64_t tile_offset, int64_t tile_step,
@@ -135,12 +183,26 @@ skycube_status skycube_dev_compact(skycube_ctx *ctx, const uint32_t *d_rows32, u
                                    int32_t *d_ext_ids, int64_t *d_offsets, int32_t *d_ids,
                                    int64_t *total_ids, void *stream);
 
+/* Partial skycube for the following skycube_dev_mdmc calls (Appendix A.2; see skycube_opts.max_level):
+ * 0 = full skycube, d' in [1, 16] = report only |delta| <= d'. */
+skycube_status skycube_ctx_set_max_level(skycube_ctx *ctx, int32_t max_level);
+
+/* HashCube (K5) from the complete tiled rows of all S+ points (the d_rows32 of skycube_dev_compact),
+ * word length w in [1, 32].  Two calls: with all four output pointers NULL it builds the HashCube in the
+ * context's workspace (d_rows32 required) and returns *n_words, *total_keys, *total_ids; then with device
+ * buffers d_word_offsets[n_words+1] (int64), d_keys[total_keys] (uint32), d_key_offsets[total_keys+1]
+ * (int64), d_ids[total_ids] (int32) it copies the result (same w; d_rows32 ignored).  Layout as
+ * skycube_hashcube; ids are point ids. */
+skycube_status skycube_dev_hashcube(skycube_ctx *ctx, const uint32_t *d_rows32, uint32_t w, int64_t *d_word_offsets,
+                                    uint32_t *d_keys, int64_t *d_key_offsets, int32_t *d_ids, int64_t *n_words,
+                                    int64_t *total_keys, int64_t *total_ids, void *stream);
+
 /* Number of kernels launched by this context since creation (for the benchmark's gpu_launches). */
 int64_t skycube_ctx_launches(const skycube_ctx *ctx);
 
 /* Work counters accumulated by the context since creation (device-side, read with a sync):
  * out8[0] K1 chunk-corner tests, [1] K1 pair tests, [2] K3 chunk-corner tests, [3] K3 pair tests,
- * [4] K3 misses (pairs that reached Alg. 3 lines 10-12), [5..7] reserved (0).  Used by the benchmark's
+ * [4] K3 misses (pairs that reached Alg. 3 lines 10-12), [5] K3 sub-chunk corner tests, [6..7] reserved (0).  Used by the benchmark's
  * roofline (algorithmic work actually required after pruning). */
 skycube_status skycube_ctx_counters(const skycube_ctx *ctx, int64_t *out8);
 

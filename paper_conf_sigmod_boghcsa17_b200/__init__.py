@@ -24,7 +24,8 @@ EXPORTED = (
     "skycube_build", "skycube_build_ex", "skycube_free", "skycube_strerror", "skycube_last_error",
     "skycube_ctx_create", "skycube_ctx_destroy", "skycube_dev_prepare", "skycube_dev_prefilter",
     "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
-    "skycube_ctx_info", "skycube_ctx_counters",
+    "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_free",
+    "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube",
 )
 
 
@@ -49,7 +50,17 @@ class Result(ctypes.Structure):
 
 
 class Opts(ctypes.Structure):
-    _fields_ = [("num_gpus", ctypes.c_int32), ("device", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+    _fields_ = [("num_gpus", ctypes.c_int32), ("device", ctypes.c_int32), ("flags", ctypes.c_uint32),
+                ("max_level", ctypes.c_int32)]
+
+
+class HashCube(ctypes.Structure):
+    _fields_ = [
+        ("d", ctypes.c_int32), ("w", ctypes.c_uint32), ("n", ctypes.c_int64), ("n_ext", ctypes.c_int64),
+        ("n_words", ctypes.c_int64), ("total_keys", ctypes.c_int64), ("total_ids", ctypes.c_int64),
+        ("word_offsets", ctypes.POINTER(ctypes.c_int64)), ("keys", ctypes.POINTER(ctypes.c_uint32)),
+        ("key_offsets", ctypes.POINTER(ctypes.c_int64)), ("ids", ctypes.POINTER(ctypes.c_int32)),
+    ]
 
 
 class Stats(ctypes.Structure):
@@ -93,9 +104,18 @@ def lib():
         L.skycube_ctx_launches.restype = I64
         L.skycube_ctx_info.argtypes = [P, ctypes.POINTER(I64), ctypes.POINTER(U32), ctypes.POINTER(U32)]
         L.skycube_ctx_counters.argtypes = [P, P]
+        L.skycube_build_hashcube.argtypes = [P, I64, I32, U32, ctypes.POINTER(Opts), ctypes.POINTER(HashCube),
+                                             ctypes.POINTER(Stats)]
+        L.skycube_hashcube_free.argtypes = [ctypes.POINTER(HashCube)]
+        L.skycube_hashcube_free.restype = None
+        L.skycube_hashcube_query.argtypes = [ctypes.POINTER(HashCube), U32, P, ctypes.POINTER(I64)]
+        L.skycube_ctx_set_max_level.argtypes = [P, I32]
+        L.skycube_dev_hashcube.argtypes = [P, P, U32, P, P, P, P, ctypes.POINTER(I64), ctypes.POINTER(I64),
+                                           ctypes.POINTER(I64), P]
         for f in ("skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
-                  "skycube_ctx_info", "skycube_ctx_counters"):
+                  "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_query",
+                  "skycube_ctx_set_max_level", "skycube_dev_hashcube"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -178,13 +198,14 @@ class RawResult:
 
 
 def skycube_build_raw(points: np.ndarray, *, device: int = 0, lists: bool = True, ext_membership: bool = False,
-                      stats: bool = False) -> RawResult:
-    """Call skycube_build_ex on a host (n, d) float32 array; returns the owning RawResult."""
+                      stats: bool = False, max_level: int = 0) -> RawResult:
+    """Call skycube_build_ex on a host (n, d) float32 array; returns the owning RawResult.
+    max_level = d' > 0 computes the partial skycube (|delta| <= d' only, Appendix A.2)."""
     pts = np.ascontiguousarray(points, dtype=np.float32)
     if pts.ndim != 2:
         raise ValueError("points must be (n, d)")
     n, d = pts.shape
-    opts = Opts(1, device, (0 if lists else NO_LISTS) | (EXT_MEMBERSHIP if ext_membership else 0))
+    opts = Opts(1, device, (0 if lists else NO_LISTS) | (EXT_MEMBERSHIP if ext_membership else 0), max_level)
     res = Result()
     st = Stats() if stats else None
     _check(lib().skycube_build_ex(pts.ctypes.data_as(ctypes.c_void_p) if n else None, n, d, ctypes.byref(opts),
@@ -204,6 +225,78 @@ def skycube_build(points: np.ndarray, **kw) -> dict:
         em = r.ext_membership()
         if em is not None:
             out["ext_rows"] = em.copy()
+        if r.stats is not None:
+            out["stats"] = r.stats
+        return out
+
+
+class RawHashCube:
+    """Owns a skycube_hashcube (pinned host buffers); views are valid until close()."""
+
+    def __init__(self, hc: HashCube, stats: Stats | None):
+        self._hc = hc
+        self.stats = stats.as_dict() if stats is not None else None
+
+    def arrays(self) -> dict:
+        h = self._hc
+        return {"word_offsets": _view(h.word_offsets, h.n_words + 1, np.int64),
+                "keys": _view(h.keys, h.total_keys, np.uint32),
+                "key_offsets": _view(h.key_offsets, h.total_keys + 1, np.int64),
+                "ids": _view(h.ids, h.total_ids, np.int32)}
+
+    def query(self, delta: int) -> np.ndarray:
+        """S_delta(P) ascending, through skycube_hashcube_query (L1280)."""
+        cnt = ctypes.c_int64()
+        _check(lib().skycube_hashcube_query(ctypes.byref(self._hc), delta, None, ctypes.byref(cnt)))
+        out = np.zeros(max(cnt.value, 1), np.int32)
+        _check(lib().skycube_hashcube_query(ctypes.byref(self._hc), delta, out.ctypes.data_as(ctypes.c_void_p),
+                                            ctypes.byref(cnt)))
+        return out[:cnt.value]
+
+    @property
+    def n_ext(self):
+        return self._hc.n_ext
+
+    def close(self):
+        if self._hc is not None:
+            lib().skycube_hashcube_free(ctypes.byref(self._hc))
+            self._hc = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def skycube_build_hashcube_raw(points: np.ndarray, w: int = 32, *, device: int = 0, max_level: int = 0,
+                               stats: bool = False) -> RawHashCube:
+    """Call skycube_build_hashcube (HashCube output, Appendix B.1) on a host (n, d) float32 array."""
+    pts = np.ascontiguousarray(points, dtype=np.float32)
+    if pts.ndim != 2:
+        raise ValueError("points must be (n, d)")
+    n, d = pts.shape
+    opts = Opts(1, device, 0, max_level)
+    hc = HashCube()
+    st = Stats() if stats else None
+    _check(lib().skycube_build_hashcube(pts.ctypes.data_as(ctypes.c_void_p) if n else None, n, d, w,
+                                        ctypes.byref(opts), ctypes.byref(hc),
+                                        ctypes.byref(st) if st is not None else None))
+    return RawHashCube(hc, st)
+
+
+def skycube_build_hashcube(points: np.ndarray, w: int = 32, **kw) -> dict:
+    """HashCube of a host (n, d) float32 array, copied into numpy arrays (word_offsets, keys, key_offsets,
+    ids) plus n_ext."""
+    with skycube_build_hashcube_raw(points, w, **kw) as r:
+        out = {k: v.copy() for k, v in r.arrays().items()}
+        out["n_ext"] = r.n_ext
         if r.stats is not None:
             out["stats"] = r.stats
         return out
@@ -251,6 +344,21 @@ class Context:
         _check(lib().skycube_dev_compact(self._h, d_rows32, d_membership or None, d_ext_ids or None,
                                          d_offsets or None, d_ids or None, ctypes.byref(tot), stream or None))
         return tot.value
+
+    def set_max_level(self, max_level: int):
+        _check(lib().skycube_ctx_set_max_level(self._h, max_level))
+
+    def hashcube(self, d_rows32: int, w: int, stream: int = 0):
+        """Build the HashCube in the context workspace: returns (n_words, total_keys, total_ids)."""
+        nw, nk, ni = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        _check(lib().skycube_dev_hashcube(self._h, d_rows32, w, None, None, None, None, ctypes.byref(nw),
+                                          ctypes.byref(nk), ctypes.byref(ni), stream or None))
+        return nw.value, nk.value, ni.value
+
+    def hashcube_copy(self, w: int, d_word_offsets: int, d_keys: int, d_key_offsets: int, d_ids: int,
+                      stream: int = 0):
+        _check(lib().skycube_dev_hashcube(self._h, None, w, d_word_offsets, d_keys, d_key_offsets, d_ids,
+                                          None, None, None, stream or None))
 
     @property
     def launches(self) -> int:

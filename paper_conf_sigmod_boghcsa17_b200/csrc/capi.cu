@@ -2,6 +2,7 @@
 // pinned host-memory pool for results, phase orchestration on one stream, and per-phase CUDA-event
 // statistics.  Every compute step runs in the kernels of prep.cu / k1_prefilter.cu / k3_mdmc.cu /
 // k4_compact.cu; there is no CPU fallback: without an sm_100 device every call fails with ENODEV.
+#include <algorithm>
 #include <chrono>
 #include <cstring>
 #include <map>
@@ -94,9 +95,11 @@ void check_device(int device) {
         throw sky::Error{SKYCUBE_ENODEV, "no CUDA device visible"};
     }
     if (device < 0 || device >= count) throw sky::Error{SKYCUBE_ENODEV, "device ordinal out of range"};
-    cudaDeviceProp prop;
-    SKY_CUDA(cudaGetDeviceProperties(&prop, device));
-    if (prop.major != 10) throw sky::Error{SKYCUBE_ENODEV, std::string("not an sm_100 device: ") + prop.name};
+    // cudaDeviceGetAttribute, not cudaGetDeviceProperties: the latter queries every property and can
+    // cost tens of milliseconds per call (it sat inside the e2e timed region)
+    int major = 0;
+    SKY_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device));
+    if (major != 10) throw sky::Error{SKYCUBE_ENODEV, "not an sm_100 device (compute capability " + std::to_string(major) + ".x)"};
     SKY_CUDA(cudaSetDevice(device));
 }
 
@@ -131,6 +134,42 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
     cudaEventElapsedTime(&ms, a, b);
     return ms;
 }
+
+// H2D of the points, then K0/K2 prepare, K1 prefilter, S+ install and K3 MDMC into x->rows32 (tiled
+// rows of the S+ points).  Events: ev[0] before H2D, ev[1] after H2D, ev[2] after prepare, ev[3] after
+// the prefilter, ev[4] after MDMC.
+void device_rows(skycube_ctx *x, const float *points, int64_t n, int d, int max_level, bool want_ext,
+                 cudaStream_t s, cudaEvent_t *ev) {
+    sky::Ctx &c = x->c;
+    const uint32_t W = sky::words_per_row(d);
+    x->input.ensure(sizeof(float) * n * d);
+    SKY_CUDA(cudaEventRecord(ev[0], s));
+    SKY_CUDA(cudaMemcpyAsync(x->input.p, points, sizeof(float) * n * d, cudaMemcpyHostToDevice, s));
+    SKY_CUDA(cudaEventRecord(ev[1], s));
+    sky::prep_run(c, x->input.as<float>(), n, d, s);
+    SKY_CUDA(cudaEventRecord(ev[2], s));
+    x->ext8.ensure(n);
+    sky::prefilter_run(c, 0, 1, x->ext8.as<uint8_t>(), s);
+    sky::ext_build(c, x->ext8.as<uint8_t>(), s);
+    SKY_CUDA(cudaEventRecord(ev[3], s));
+    const int64_t m = c.m;
+    const size_t rows_words = (size_t)sky::ceil_div(m > 0 ? m : 1, 32) * 32 * W;
+    x->rows32.ensure(sizeof(uint32_t) * rows_words);
+    if (want_ext) x->ext_rows32.ensure(sizeof(uint32_t) * rows_words);
+    c.max_level = max_level;
+    sky::mdmc_run(c, 0, m, x->rows32.as<uint32_t>(), want_ext ? x->ext_rows32.as<uint32_t>() : nullptr, s);
+    SKY_CUDA(cudaEventRecord(ev[4], s));
+}
+
+struct Events {
+    cudaEvent_t e[9];
+    Events() {
+        for (auto &v : e) SKY_CUDA(cudaEventCreate(&v));
+    }
+    ~Events() {
+        for (auto &v : e) cudaEventDestroy(v);
+    }
+};
 
 }  // namespace
 
@@ -171,6 +210,8 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
     if (n > 0 && !points) return fail(SKYCUBE_EINVAL, "points == NULL");
     const uint32_t flags = opts ? opts->flags : 0u;
     const int device = opts ? opts->device : 0;
+    const int max_level = opts ? opts->max_level : 0;
+    if (max_level < 0 || max_level > d) return fail(SKYCUBE_EINVAL, "max_level must be in [0, d]");
     std::lock_guard<std::mutex> lk(g_mutex);
     const auto t0 = std::chrono::steady_clock::now();
     skycube_result r;
@@ -186,6 +227,7 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
         else check_device(device);
         sky::Ctx &c = x->c;
         const int64_t launches0 = c.L.count;
+        const bool want_ext = (flags & SKYCUBE_EXT_MEMBERSHIP) != 0;
         if (n == 0) {
             if (!(flags & SKYCUBE_NO_LISTS)) {
                 r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
@@ -194,29 +236,10 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
             return;
         }
         cudaStream_t s = nullptr;
-        cudaEvent_t ev[9];
-        for (auto &e : ev) SKY_CUDA(cudaEventCreate(&e));
-        struct EvGuard {
-            cudaEvent_t *e;
-            ~EvGuard() { for (int i = 0; i < 9; i++) cudaEventDestroy(e[i]); }
-        } eg{ev};
-        x->input.ensure(sizeof(float) * n * d);
-        SKY_CUDA(cudaEventRecord(ev[0], s));
-        SKY_CUDA(cudaMemcpyAsync(x->input.p, points, sizeof(float) * n * d, cudaMemcpyHostToDevice, s));
-        SKY_CUDA(cudaEventRecord(ev[1], s));
-        sky::prep_run(c, x->input.as<float>(), n, d, s);
-        SKY_CUDA(cudaEventRecord(ev[2], s));
-        x->ext8.ensure(n);
-        sky::prefilter_run(c, 0, 1, x->ext8.as<uint8_t>(), s);
-        sky::ext_build(c, x->ext8.as<uint8_t>(), s);
-        SKY_CUDA(cudaEventRecord(ev[3], s));
+        Events evs;
+        cudaEvent_t *ev = evs.e;
+        device_rows(x, points, n, d, max_level, want_ext, s, ev);
         const int64_t m = c.m;
-        const size_t rows_words = (size_t)sky::ceil_div(m > 0 ? m : 1, 32) * 32 * W;
-        x->rows32.ensure(sizeof(uint32_t) * rows_words);
-        const bool want_ext = (flags & SKYCUBE_EXT_MEMBERSHIP) != 0;
-        if (want_ext) x->ext_rows32.ensure(sizeof(uint32_t) * rows_words);
-        sky::mdmc_run(c, 0, m, x->rows32.as<uint32_t>(), want_ext ? x->ext_rows32.as<uint32_t>() : nullptr, s);
-        SKY_CUDA(cudaEventRecord(ev[4], s));
         x->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
         sky::compact_membership(c, x->rows32.as<uint32_t>(), x->membership.as<uint32_t>(), s);
         int64_t total = 0;
@@ -281,6 +304,114 @@ skycube_status skycube_build(const float *points, int64_t n, int32_t d, skycube_
     return skycube_build_ex(points, n, d, nullptr, out, nullptr);
 }
 
+// ------------------------------------------------------------------------------ HashCube (NEXT-1/4)
+void skycube_hashcube_free(skycube_hashcube *hc) {
+    if (!hc) return;
+    g_pool.put(hc->word_offsets);
+    g_pool.put(hc->keys);
+    g_pool.put(hc->key_offsets);
+    g_pool.put(hc->ids);
+    std::memset(hc, 0, sizeof(*hc));
+}
+
+skycube_status skycube_build_hashcube(const float *points, int64_t n, int32_t d, uint32_t w, const skycube_opts *opts,
+                                      skycube_hashcube *out, skycube_stats *stats) {
+    if (!out) return fail(SKYCUBE_EINVAL, "out == NULL");
+    std::memset(out, 0, sizeof(*out));
+    if (stats) std::memset(stats, 0, sizeof(*stats));
+    if (d < 1 || d > 16) return fail(SKYCUBE_EINVAL, "d must be in [1, 16]");
+    if (w < 1 || w > 32) return fail(SKYCUBE_EINVAL, "w must be in [1, 32]");
+    if (n < 0 || n > INT32_MAX) return fail(SKYCUBE_EINVAL, "n must be in [0, INT32_MAX]");
+    if (n > 0 && !points) return fail(SKYCUBE_EINVAL, "points == NULL");
+    const int device = opts ? opts->device : 0;
+    const int max_level = opts ? opts->max_level : 0;
+    if (max_level < 0 || max_level > d) return fail(SKYCUBE_EINVAL, "max_level must be in [0, d]");
+    std::lock_guard<std::mutex> lk(g_mutex);
+    const auto t0 = std::chrono::steady_clock::now();
+    skycube_hashcube r;
+    std::memset(&r, 0, sizeof(r));
+    skycube_status st = guarded([&] {
+        r.d = d;
+        r.w = w;
+        r.n = n;
+        r.n_words = sky::hashcube_words(d, w);
+        skycube_ctx *&x = g_ctx[device];
+        if (!x) x = new_ctx(device);
+        else check_device(device);
+        sky::Ctx &c = x->c;
+        const int64_t launches0 = c.L.count;
+        if (n == 0) {
+            r.word_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (r.n_words + 1));
+            std::memset(r.word_offsets, 0, sizeof(int64_t) * (r.n_words + 1));
+            r.key_offsets = (int64_t *)g_pool.get(sizeof(int64_t));
+            r.key_offsets[0] = 0;
+            return;
+        }
+        cudaStream_t s = nullptr;
+        Events evs;
+        cudaEvent_t *ev = evs.e;
+        device_rows(x, points, n, d, max_level, false, s, ev);
+        sky::hashcube_build(c, x->rows32.as<uint32_t>(), w, s);
+        SKY_CUDA(cudaEventRecord(ev[5], s));
+        const sky::HashCubeState &h = c.hc;
+        r.n_ext = c.m;
+        r.total_keys = h.nkeys;
+        r.total_ids = h.nvalid;
+        r.word_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (h.nwords + 1));
+        r.keys = (uint32_t *)g_pool.get(sizeof(uint32_t) * (h.nkeys > 0 ? h.nkeys : 1));
+        r.key_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (h.nkeys + 1));
+        r.ids = (int32_t *)g_pool.get(sizeof(int32_t) * (h.nvalid > 0 ? h.nvalid : 1));
+        SKY_CUDA(cudaMemcpyAsync(r.word_offsets, h.woff.p, sizeof(int64_t) * (h.nwords + 1), cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaMemcpyAsync(r.key_offsets, h.koff.p, sizeof(int64_t) * (h.nkeys + 1), cudaMemcpyDeviceToHost, s));
+        if (h.nkeys) SKY_CUDA(cudaMemcpyAsync(r.keys, h.keys32.p, sizeof(uint32_t) * h.nkeys, cudaMemcpyDeviceToHost, s));
+        if (h.nvalid) SKY_CUDA(cudaMemcpyAsync(r.ids, h.vals.p, sizeof(int32_t) * h.nvalid, cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaEventRecord(ev[6], s));
+        SKY_CUDA(cudaStreamSynchronize(s));
+        SKY_CUDA(cudaGetLastError());
+        if (stats) {
+            stats->ms_h2d = ev_ms(ev[0], ev[1]);
+            stats->ms_sort = ev_ms(ev[1], ev[2]);
+            stats->ms_prefilter = ev_ms(ev[2], ev[3]);
+            stats->ms_mdmc = ev_ms(ev[3], ev[4]);
+            stats->ms_compact = ev_ms(ev[4], ev[5]);
+            stats->ms_d2h = ev_ms(ev[5], ev[6]);
+            stats->n_ext = c.m;
+            stats->pairs = c.m * (c.m > 0 ? c.m - 1 : 0);
+            stats->total_ids = h.nvalid;
+            stats->kernel_launches = (int32_t)(c.L.count - launches0);
+        }
+    });
+    if (st != SKYCUBE_OK) {
+        skycube_hashcube_free(&r);
+        return st;
+    }
+    if (stats)
+        stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = r;
+    return SKYCUBE_OK;
+}
+
+skycube_status skycube_hashcube_query(const skycube_hashcube *hc, uint32_t delta, int32_t *ids, int64_t *count) {
+    if (!hc || !count) return fail(SKYCUBE_EINVAL, "NULL argument");
+    if (hc->d < 1 || hc->d > 16 || hc->w < 1 || hc->w > 32 || !hc->word_offsets || !hc->key_offsets)
+        return fail(SKYCUBE_EINVAL, "not a HashCube built by skycube_build_hashcube");
+    if (delta == 0 || delta >= (1u << hc->d)) return fail(SKYCUBE_EINVAL, "delta must be in [1, 2^d - 1]");
+    return guarded([&] {
+        // L1280 (reading Q6): the lists of h_{(delta-1)/w} whose key has bit (delta-1) % w unset
+        const int64_t k = (int64_t)(delta - 1) / hc->w;
+        const uint32_t b = (delta - 1) % hc->w;
+        int64_t cnt = 0;
+        for (int64_t u = hc->word_offsets[k]; u < hc->word_offsets[k + 1]; u++) {
+            if ((hc->keys[u] >> b) & 1u) continue;
+            const int64_t lo = hc->key_offsets[u], hi = hc->key_offsets[u + 1];
+            if (ids) std::memcpy(ids + cnt, hc->ids + lo, sizeof(int32_t) * (size_t)(hi - lo));
+            cnt += hi - lo;
+        }
+        if (ids) std::sort(ids, ids + cnt);  // ascending, like the lattice (reading Q12)
+        *count = cnt;
+    });
+}
+
 // ------------------------------------------------------------------------------ device-level API
 skycube_status skycube_ctx_create(int32_t device, skycube_ctx **ctx) {
     if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
@@ -299,6 +430,7 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
                            &c.scan64_tmp, &c.chunks_all, &c.chunks_ext, &c.supers_all, &c.counters, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
                            &ctx->membership, &ctx->offsets, &ctx->ids})
         b->release();
+    c.hc.release();
     delete ctx;
 }
 
@@ -356,6 +488,42 @@ skycube_status skycube_dev_mdmc(skycube_ctx *ctx, int64_t j_begin, int64_t j_end
     return guarded([&] {
         SKY_CUDA(cudaSetDevice(ctx->c.device));
         sky::mdmc_run(ctx->c, j_begin, j_end, d_rows32, d_ext_rows32, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_ctx_set_max_level(skycube_ctx *ctx, int32_t max_level) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (max_level < 0 || max_level > 16) return fail(SKYCUBE_EINVAL, "max_level must be in [0, 16]");
+    ctx->c.max_level = max_level;
+    return SKYCUBE_OK;
+}
+
+skycube_status skycube_dev_hashcube(skycube_ctx *ctx, const uint32_t *d_rows32, uint32_t w, int64_t *d_word_offsets,
+                                    uint32_t *d_keys, int64_t *d_key_offsets, int32_t *d_ids, int64_t *n_words,
+                                    int64_t *total_keys, int64_t *total_ids, void *stream) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (w < 1 || w > 32) return fail(SKYCUBE_EINVAL, "w must be in [1, 32]");
+    const bool copy = d_word_offsets || d_keys || d_key_offsets || d_ids;
+    if (copy && !(d_word_offsets && d_key_offsets && d_keys && d_ids))
+        return fail(SKYCUBE_EINVAL, "all four output buffers are needed");
+    if (!copy && !d_rows32) return fail(SKYCUBE_EINVAL, "d_rows32 == NULL");
+    return guarded([&] {
+        sky::Ctx &c = ctx->c;
+        SKY_CUDA(cudaSetDevice(c.device));
+        cudaStream_t s = (cudaStream_t)stream;
+        sky::HashCubeState &h = c.hc;
+        if (!copy) {
+            sky::hashcube_build(c, d_rows32, w, s);
+        } else {
+            if (!h.built || h.w != w) throw sky::Error{SKYCUBE_EINVAL, "no HashCube with this w was built"};
+            SKY_CUDA(cudaMemcpyAsync(d_word_offsets, h.woff.p, sizeof(int64_t) * (h.nwords + 1), cudaMemcpyDeviceToDevice, s));
+            SKY_CUDA(cudaMemcpyAsync(d_key_offsets, h.koff.p, sizeof(int64_t) * (h.nkeys + 1), cudaMemcpyDeviceToDevice, s));
+            if (h.nkeys) SKY_CUDA(cudaMemcpyAsync(d_keys, h.keys32.p, sizeof(uint32_t) * h.nkeys, cudaMemcpyDeviceToDevice, s));
+            if (h.nvalid) SKY_CUDA(cudaMemcpyAsync(d_ids, h.vals.p, sizeof(int32_t) * h.nvalid, cudaMemcpyDeviceToDevice, s));
+        }
+        if (n_words) *n_words = h.nwords;
+        if (total_keys) *total_keys = h.nkeys;
+        if (total_ids) *total_ids = h.nvalid;
     });
 }
 

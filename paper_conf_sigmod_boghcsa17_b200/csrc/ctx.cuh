@@ -31,6 +31,23 @@ struct DevBuf {
     }
 };
 
+// HashCube of the last skycube_dev_hashcube / skycube_build_hashcube call (K5, k5_hashcube.cu)
+struct HashCubeState {
+    bool built = false;
+    uint32_t w = 0;
+    int64_t nwords = 0, nvalid = 0, nkeys = 0;
+    DevBuf keys, vals, keys_alt, vals_alt, counts, scan_tmp, nvalid_dev;  // items (word, key) -> id, sorted
+    DevBuf ukeys;   // u64 [nkeys]   distinct composites (k << w) | key
+    DevBuf keys32;  // u32 [nkeys]   keys
+    DevBuf koff;    // i64 [nkeys+1] first item of each key (ids = vals[koff[u] .. koff[u+1]))
+    DevBuf woff;    // i64 [nwords+1] first key of each word
+    void release() {
+        for (DevBuf *b : {&keys, &vals, &keys_alt, &vals_alt, &counts, &scan_tmp, &nvalid_dev, &ukeys, &keys32, &koff, &woff})
+            b->release();
+        built = false;
+    }
+};
+
 struct Ctx {
     int device = 0;
     int num_sms = 148;
@@ -42,6 +59,7 @@ struct Ctx {
     uint32_t exact_mask = 0;    // bit i <=> the codes of dimension i are injective (dense ranks)
     uint32_t R[kMaxD] = {0};    // distinct values per dimension
     int64_t m = 0;              // |S+(P)|
+    int max_level = 0;          // partial skycube (Appendix A.2): report only |delta| <= max_level (0 = d)
     bool prepared = false, ext_ready = false;
     // preparation (all n points)
     DevBuf ord;         // u32 [n*d]   order-preserving keys, id order
@@ -74,6 +92,7 @@ struct Ctx {
     DevBuf lat_counts;  // u64 [2^d * nchunks]
     DevBuf counters;    // u64 [8]: K1 box tests, K1 pair tests, K3 box tests, K3 pair tests, K3 misses
     DevBuf scan64_tmp;
+    HashCubeState hc;
 };
 
 // prep.cu
@@ -87,6 +106,9 @@ void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32
 void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cudaStream_t st);
 void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
                      cudaStream_t st);
+// k5_hashcube.cu
+int64_t hashcube_words(int d, uint32_t w);
+void hashcube_build(Ctx &c, const uint32_t *rows32, uint32_t w, cudaStream_t st);
 
 constexpr int64_t kQPad = 1024;      // competitor stream padded to whole MDMC tiles
 constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole

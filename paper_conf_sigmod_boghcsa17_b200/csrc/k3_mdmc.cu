@@ -208,6 +208,17 @@ __device__ __forceinline__ void expand(uint32_t *st, uint32_t *tr, int trs, uint
     });
 }
 
+// Partial skycube (Appendix A.2; reading P1): bits b of a membership word whose subspace
+// 32w + b has at most k dimensions in the low five (k = d' - |w|, w the word index = dimensions 5..d-1).
+__device__ __forceinline__ uint32_t level_pattern(int k) {
+    if (k < 0) return 0u;
+    uint32_t r = 0;
+#pragma unroll
+    for (int b = 0; b < 32; b++)
+        if (__popc(b) <= k) r |= 1u << b;
+    return r;
+}
+
 // CW words from a 16-byte aligned row (CW even): LDS.128 / LDS.64 instead of CW scalar loads.
 template <int CW>
 __device__ __forceinline__ void load_row(const uint32_t *p, uint32_t *w) {
@@ -230,7 +241,7 @@ template <int D, int MODE>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
-    int64_t j_end, uint32_t inexact, int tpc, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
+    int64_t j_end, uint32_t inexact, int tpc, int max_level, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
     uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
@@ -426,11 +437,12 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             } else {
                 v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
             }
-            uint32_t row = ~v & G::kRowMask;
+            const uint32_t lvl = max_level > 0 ? level_pattern(max_level - __popc(w)) : 0xffffffffu;
+            uint32_t row = ~v & G::kRowMask & lvl;
             if (w == 0) row &= ~1u;
             out[w * 32] = row;
             if (ext_rows32) {
-                uint32_t er = ~st[w] & G::kRowMask;
+                uint32_t er = ~st[w] & G::kRowMask & lvl;
                 if (w == 0) er &= ~1u;
                 ext_rows32[(jt >> 5) * (G::WB * 32) + w * 32 + (jt & 31)] = er;
             }
@@ -450,7 +462,8 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_mdmc_kernel<D, MODE><<<blocks, (kWarps + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc, rows32,
+        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc,
+        (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32,
         c.tie.as<uint32_t>(), ext_rows32, c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();

@@ -100,9 +100,12 @@ class DeviceSkycube:
     def launches(self) -> int:
         return self.ctx.launches
 
-    def build(self, pts: torch.Tensor, lists: bool = True, membership: bool = True, events: dict | None = None):
+    def build(self, pts: torch.Tensor, lists: bool = True, membership: bool = True, events: dict | None = None,
+              hashcube_w: int = 0, max_level: int = 0):
         """pts: (n, d) float32 CUDA tensor (resident).  Returns dict of device tensors:
-        n_ext, rows32 (tiled rows of S+), ext_ids, membership [n, W] (optional), offsets, ids."""
+        n_ext, rows32 (tiled rows of S+), ext_ids, membership [n, W] (optional), offsets, ids, and with
+        hashcube_w > 0 the HashCube (K5, Appendix B.1) as hashcube = {word_offsets, keys, key_offsets, ids}.
+        max_level = d' > 0: partial skycube (Appendix A.2), only |delta| <= d' reported."""
         assert pts.is_cuda and pts.dtype == torch.float32 and pts.dim() == 2
         pts = pts.contiguous()
         n, d = pts.shape
@@ -124,6 +127,7 @@ class DeviceSkycube:
         rec("t2")
         rows32 = torch.empty(rows_buffer_words(m, d, world), dtype=torch.int32, device=self.device)
         j0, j1 = task_range(m, world, rank)
+        self.ctx.set_max_level(max_level)
         if j1 > j0:
             self.ctx.mdmc(rows32.data_ptr(), j0, j1, 0, sp)
         rec("t3")
@@ -142,6 +146,17 @@ class DeviceSkycube:
             out["offsets"] = offsets
             out["ids"] = ids[:total]
             out["total_ids"] = total
+        if hashcube_w:
+            nw, nk, ni = self.ctx.hashcube(rows32.data_ptr(), hashcube_w, sp)
+            hc = {"word_offsets": torch.empty(nw + 1, dtype=torch.int64, device=self.device),
+                  "keys": torch.empty(max(nk, 1), dtype=torch.int32, device=self.device),
+                  "key_offsets": torch.empty(nk + 1, dtype=torch.int64, device=self.device),
+                  "ids": torch.empty(max(ni, 1), dtype=torch.int32, device=self.device)}
+            self.ctx.hashcube_copy(hashcube_w, hc["word_offsets"].data_ptr(), hc["keys"].data_ptr(),
+                                   hc["key_offsets"].data_ptr(), hc["ids"].data_ptr(), sp)
+            hc["keys"] = hc["keys"][:nk]
+            hc["ids"] = hc["ids"][:ni]
+            out["hashcube"] = hc
         rec("t4")
         return out
 

@@ -76,3 +76,44 @@ def test_no_cpu_fallback_without_gpu(lib):
     st = lib.skycube_build(pts.ctypes.data_as(ctypes.c_void_p), 4, 3, ctypes.byref(res))
     assert st == sky.ENODEV
     assert b"device" in lib.skycube_last_error()
+
+
+def test_hashcube_and_partial_validation_without_gpu(lib):
+    pts = np.zeros((4, 3), np.float32)
+    p = pts.ctypes.data_as(ctypes.c_void_p)
+    hc = sky.HashCube()
+    assert lib.skycube_build_hashcube(p, 4, 3, 0, None, ctypes.byref(hc), None) == sky.EINVAL
+    assert lib.skycube_build_hashcube(p, 4, 3, 33, None, ctypes.byref(hc), None) == sky.EINVAL
+    assert lib.skycube_build_hashcube(p, 4, 17, 32, None, ctypes.byref(hc), None) == sky.EINVAL
+    opts = sky.Opts(1, 0, 0, 4)  # max_level > d
+    res = sky.Result()
+    assert lib.skycube_build_ex(p, 4, 3, ctypes.byref(opts), ctypes.byref(res), None) == sky.EINVAL
+    cnt = ctypes.c_int64()
+    assert lib.skycube_hashcube_query(ctypes.byref(sky.HashCube()), 1, None, ctypes.byref(cnt)) == sky.EINVAL
+    lib.skycube_hashcube_free(ctypes.byref(hc))  # safe on a zeroed struct
+
+
+def test_hashcube_query_host_logic_fig1b(lib):
+    """The read path (skycube_hashcube_query, host code) on the Fig. 1b HashCube built by the oracle."""
+    import json
+    import oracle
+    from oracle import hashcube as hco
+    gold = json.load(open(os.path.join(ROOT, "tests", "golden", "flights.json")))
+    x = np.array(gold["points"], np.float32)
+    for w in (4, 1, 3, 32):
+        a = hco.hashcube(oracle.rows_a(x, with_ext=False), 3, w)
+        hc = sky.HashCube()
+        hc.d, hc.w, hc.n, hc.n_words = 3, w, 5, hco.n_words(3, w)
+        hc.total_keys, hc.total_ids = a["keys"].size, a["ids"].size
+        hc.word_offsets = a["word_offsets"].ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+        hc.keys = a["keys"].ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
+        hc.key_offsets = a["key_offsets"].ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+        hc.ids = a["ids"].ctypes.data_as(ctypes.POINTER(ctypes.c_int32))
+        for delta in range(1, 8):
+            cnt = ctypes.c_int64()
+            assert lib.skycube_hashcube_query(ctypes.byref(hc), delta, None, ctypes.byref(cnt)) == sky.OK
+            out = np.zeros(max(1, cnt.value), np.int32)
+            assert lib.skycube_hashcube_query(ctypes.byref(hc), delta, out.ctypes.data_as(ctypes.c_void_p),
+                                              ctypes.byref(cnt)) == sky.OK
+            assert out[:cnt.value].tolist() == gold["lattice"][str(delta)], (w, delta)
+        assert lib.skycube_hashcube_query(ctypes.byref(hc), 8, None, ctypes.byref(cnt)) == sky.EINVAL
