@@ -49,6 +49,18 @@ def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
     return sms * 128 * sm_mhz * 1e6
 
 
+def ncu_traffic(config: str, kernel: str):
+    """dram__bytes_read.sum + dram__bytes_write.sum of one launch of `kernel` at `config`, from the committed
+    ncu --set full capture summarised in profiles/traffic.json (None if there is no capture)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            t = json.load(f)
+        e = t[config][kernel]
+        return int(e["dram_read_bytes"]) + int(e["dram_write_bytes"]), e.get("source")
+    except Exception:
+        return None, None
+
+
 def workload(cfg) -> str:
     return f"{cfg.name}: {cfg.dist} n={cfg.n} d={cfg.d} seed={cfg.seed} (datagen, Börzsönyi-style)"
 
@@ -276,6 +288,7 @@ def run_ours(args):
     ops = tests * algorithmic_ops_per_test(d)
     achieved = ops / (mdmc_ms / 1e3) / 1e12
     peak = alu_peak_ops(sm_mhz) / 1e12
+    traffic, traffic_src = ncu_traffic(args.config, "k3_mdmc") if world == 1 else (None, None)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
@@ -289,7 +302,8 @@ def run_ours(args):
         "work_per_step": work,
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
-                     "frac": achieved / peak, "traffic": None,
+                     "frac": achieved / peak, "traffic": traffic, "traffic_unit": "bytes (DRAM read+write per launch)",
+                     "traffic_source": traffic_src,
                      "kernel": "k3_mdmc", "ops_per_test": algorithmic_ops_per_test(d), "tests": tests,
                      "peak_basis": f"148 SM x 128 integer lanes/clk (ALU+FMA pipes, 1 warp-inst/SMSP/clk) x {sm_mhz:.0f} MHz "
                                    f"(median SM clock under load)"},

@@ -10,7 +10,10 @@
 //
 // CTA: 16 consumer warps, each owning 32 consecutive tree positions (one task per lane, codes in
 // registers), and one TMA producer warp streaming tiles through a ring; the warps never wait for each
-// other (only for the ring).  Per tile and warp:
+// other (only for the ring).  The producer streams only the tiles that can hold a dominator of SOME task of
+// the CTA -- tile corner < U in every dimension, U = the per-dimension maximum code of the CTA's 512 tasks
+// (consecutive in Morton order, so U is a tight upper corner) -- and publishes each streamed tile's index
+// with its ring slot, ending the stream with a sentinel.  Per streamed tile and warp:
 //   tile test   every live lane tests the tile corner (SWAR strict compare with guard bits); if none
 //               passes, the tile is done;
 //   chunk test  for each of the 16 chunks, the lanes that passed test the chunk corner; a ballot gives the
@@ -43,21 +46,24 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)TW};
     uint32_t *pV = smem + 4 * kStages + kStages * TW;  // [kTasks][CWV] task codes with guard bits
+    volatile int32_t *tile_idx = reinterpret_cast<volatile int32_t *>(pV + kTasks * CWV);  // [kStages]
+    uint32_t *ucorner = pV + kTasks * CWV + kStages;   // [kWarps][CW] upper corner of each warp's tasks
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t blk = blk_offset + (int64_t)blockIdx.x * blk_step;
     const int64_t s0 = blk * kTasks;
     const int64_t ntiles = ceil_div_dev(nchunks, kTileChunks);
 
     if (threadIdx.x == 0) ring.init(kWarps);
-    __syncthreads();
-    if (warp == kWarps) {  // producer warp: one elected lane streams tiles (16 chunk records + tile corner)
-        if (lane == 0)
-            for (int64_t t = 0; t < ntiles; t++) ring.issue2(chunks, kTileChunks * REC, supers, CWS, t);
-        return;
-    }
+    // corner test: q < p needs code(q) < code(p) on injective dimensions but only code(q) <= code(p) on
+    // the others (a bin may hold several values), so subtract 1 only in the injective lanes:
+    // corner < p  <=>  guard bits of (p - csub) - corner
+    uint32_t csub[CW];
+#pragma unroll
+    for (int k = 0; k < CW; k++)
+        csub[k] = (((inexact >> (2 * k)) & 1u) ? 0u : 1u) | (((inexact >> (2 * k + 1)) & 1u) ? 0u : 0x10000u);
     const int64_t ps = s0 + warp * 32 + lane;  // this lane's task (tree position)
-    uint32_t p[CW];
-    {
+    uint32_t p[CW], pm[CW];
+    if (warp < kWarps) {
         const uint32_t *src = chunks + (ps >> 5) * REC + (ps & 31) * CW;  // code rows of the chunk records
 #pragma unroll
         for (int k = 0; k < CW; k++) {
@@ -65,26 +71,66 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
             if (2 * k >= d) w |= 0x00007fffu;  // padding dimensions never reject
             if (2 * k + 1 >= d) w |= 0x7fff0000u;
             p[k] = w | kGuard;
+            pm[k] = p[k] - csub[k];
             pV[(warp * 32 + lane) * CWV + k] = p[k];
+            uint32_t lo = ps < n ? (w & 0xffffu) : 0u, hi = ps < n ? (w >> 16) : 0u;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                lo = max(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+                hi = max(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+            }
+            if (lane == 0) ucorner[warp * CW + k] = lo | (hi << 16);
         }
     }
-    __syncwarp();
-    // corner test: q < p needs code(q) < code(p) on injective dimensions but only code(q) <= code(p) on
-    // the others (a bin may hold several values), so subtract 1 only in the injective lanes
-    uint32_t csub[CW];
+    __syncthreads();
+    if (warp == kWarps) {
+        // producer warp: one elected lane streams only the tiles whose corner is below the CTA's upper
+        // corner U (per-dimension maximum code of its tasks) -- no other tile can hold a dominator of any
+        // task here -- and publishes each streamed tile's index with its ring slot; -1 ends the stream
+        if (lane == 0) {
+            uint32_t um[CW];
 #pragma unroll
-    for (int k = 0; k < CW; k++)
-        csub[k] = (((inexact >> (2 * k)) & 1u) ? 0u : 1u) | (((inexact >> (2 * k + 1)) & 1u) ? 0u : 0x10000u);
+            for (int k = 0; k < CW; k++) um[k] = 0;
+#pragma unroll
+            for (int w = 0; w < kWarps; w++) {
+#pragma unroll
+                for (int k = 0; k < CW; k++) {
+                    const uint32_t u = ucorner[w * CW + k];
+                    um[k] = max(um[k] & 0xffffu, u & 0xffffu) | (max(um[k] >> 16, u >> 16) << 16);
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < CW; k++) um[k] = (um[k] | kGuard) - csub[k];
+            int64_t slot = 0;
+            for (int64_t t = 0; t < ntiles; t++) {
+                const uint32_t *sc = supers + t * CWS;
+                uint32_t acc = 0xffffffffu;
+#pragma unroll
+                for (int k = 0; k < CW; k++) acc &= um[k] - __ldg(sc + k);
+                if ((acc & kGuard) != kGuard) continue;
+                ring.wait_empty(slot);
+                tile_idx[slot % kStages] = (int32_t)t;
+                ring.issue2_slot(chunks, kTileChunks * REC, supers, CWS, t, slot);
+                slot++;
+            }
+            ring.wait_empty(slot);
+            tile_idx[slot % kStages] = -1;
+            ring.arrive_full(slot);
+        }
+        return;
+    }
     uint32_t live = __ballot_sync(0xffffffffu, ps < n);  // tasks not (yet) dominated
     unsigned long long n_box = 0, n_pair = 0;
-    for (int64_t tile = 0; tile < ntiles; tile++) {
-        ring.wait(tile);
-        const uint32_t *stg = ring.stage(tile);
+    for (int64_t slot = 0;; slot++) {
+        ring.wait(slot);
+        const int64_t tile = tile_idx[slot % kStages];
+        if (tile < 0) break;
+        const uint32_t *stg = ring.stage(slot);
         uint32_t need = 0;
         if (live) {
             uint32_t acc = 0xffffffffu;
 #pragma unroll
-            for (int k = 0; k < CW; k++) acc &= p[k] - (stg[kTileChunks * REC + k] + csub[k]);  // tile corner < p
+            for (int k = 0; k < CW; k++) acc &= pm[k] - stg[kTileChunks * REC + k];  // tile corner < p
             need = __ballot_sync(0xffffffffu, ((live >> lane) & 1u) && (acc & kGuard) == kGuard);
             n_box += __popc(live);
         }
@@ -94,7 +140,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
             const uint32_t *rec = stg + ch * REC;
             uint32_t acc = 0xffffffffu;
 #pragma unroll
-            for (int k = 0; k < CW; k++) acc &= p[k] - (rec[32 * CW + k] + csub[k]);  // chunk corner < p
+            for (int k = 0; k < CW; k++) acc &= pm[k] - rec[32 * CW + k];  // chunk corner < p
             uint32_t todo = __ballot_sync(0xffffffffu, ((need >> lane) & 1u) && (acc & kGuard) == kGuard);
             n_box += __popc(need);
             if (!todo) continue;
@@ -138,8 +184,10 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
                 }
             }
         }
+        // every read of the stage has completed before it is handed back to the producer
+        __threadfence_block();
         __syncwarp();
-        if (lane == 0) ring.release(tile);
+        if (lane == 0) ring.release(slot);
     }
     if (lane == 0 && counters) {
         atomicAdd(&counters[0], n_box);
@@ -151,7 +199,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
 template <int CW>
 void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uint8_t *ext, cudaStream_t st) {
     const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * (kTileChunks * 33 * CW + ((CW + 3) & ~3)) +
-                                            (size_t)kTasks * ((CW + 3) & ~3));
+                                            (size_t)kTasks * ((CW + 3) & ~3) + kStages + (size_t)kWarps * CW);
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
     k1_prefilter_kernel<CW><<<(unsigned)nblk_mine, (kWarps + 1) * 32, smem, st>>>(

@@ -208,6 +208,23 @@ __device__ __forceinline__ void expand(uint32_t *st, uint32_t *tr, int trs, uint
     });
 }
 
+// Shared-memory word access through a 32-bit shared-window address computed once per kernel.  Plain
+// pointer accesses made the compiler re-materialise the dynamic shared base (S2UR SR_CgaCtaId + ULEA) in
+// the hot loops.  Probes are volatile: other warps OR bits into the state concurrently (any value read
+// is a sound subset of the final state).
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) { asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+// (laundered through an opaque move, or the compiler re-derives it from SR_CgaCtaId at every use)
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+    uint32_t a = (uint32_t)__cvta_generic_to_shared(p);
+    asm volatile("mov.b32 %0, %0;" : "+r"(a));
+    return a;
+}
+
 // Partial skycube (Appendix A.2; reading P1): bits b of a membership word whose subspace
 // 32w + b has at most k dimensions in the low five (k = d' - |w|, w the word index = dimensions 5..d-1).
 __device__ __forceinline__ uint32_t level_pattern(int k) {
@@ -237,6 +254,53 @@ __device__ __forceinline__ void load_row(const uint32_t *p, uint32_t *w) {
     }
 }
 
+// The same from a 32-bit shared address (read-only task codes: plain asm, free to schedule).
+template <int CW>
+__device__ __forceinline__ void load_row_s(uint32_t a, uint32_t *w) {
+#pragma unroll
+    for (int k = 0; k + 4 <= CW; k += 4)
+        asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+            : "=r"(w[k]), "=r"(w[k + 1]), "=r"(w[k + 2]), "=r"(w[k + 3])
+            : "r"(a + 4u * k));
+    if (CW % 4) asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(w[CW & ~3]), "=r"(w[(CW & ~3) + 1]) : "r"(a + 4u * (CW & ~3)));
+}
+
+// Epilogue of both K3 designs: B_{p notin S} -> membership row (its complement; bit 0, the empty subspace,
+// is never a member), written in the tiled layout (group of 32 tasks, word-major).
+template <int D, int MODE>
+__device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, int nt, int warp, int lane, int max_level,
+                                           uint32_t *__restrict__ rows32, const uint32_t *__restrict__ tie32,
+                                           uint32_t *__restrict__ ext_rows32) {
+    using G = Geo<D>;
+    using C = GeoK3<D, MODE>;
+    constexpr bool TIES = MODE == kModeSmemTie;
+    for (int t = warp; t < nt; t += kWarps) {
+        const int64_t jt = j0 + t;
+        const uint32_t *st = state + t * C::PS;
+        uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        const uint32_t *trg = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        for (int w = lane; w < G::WB; w += 32) {
+            uint32_t v;
+            if (MODE == kModeDims) {  // p dominated in delta <=> delta in D_i for some i in delta
+                v = 0;
+#pragma unroll
+                for (int i = 0; i < D; i++) v |= st[(1 + i) * G::WB + w] & dim_in_word(i, w);
+            } else {
+                v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+            }
+            const uint32_t lvl = max_level > 0 ? level_pattern(max_level - __popc(w)) : 0xffffffffu;
+            uint32_t row = ~v & G::kRowMask & lvl;
+            if (w == 0) row &= ~1u;
+            out[w * 32] = row;
+            if (ext_rows32) {
+                uint32_t er = ~st[w] & G::kRowMask & lvl;
+                if (w == 0) er &= ~1u;
+                ext_rows32[(jt >> 5) * (G::WB * 32) + w * 32 + (jt & 31)] = er;
+            }
+        }
+    }
+}
+
 template <int D, int MODE>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
@@ -257,6 +321,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint32_t *wq = zm + tpc + warp * C::QW;    // per-warp queue of opened tasks (<= 3 + 32 entries)
     uint32_t *iq = wq + 40;                    // per-warp queue of opened (task, sub-chunk) items (<= 7 + 32)
+    const uint32_t st_s = smem_addr(state), wq_s = smem_addr(wq), iq_s = smem_addr(iq), pV_s = smem_addr(pV);
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
@@ -316,22 +381,21 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         if (lane == 0) ring.release(tile);
         const int64_t c = tile * kWarps + warp;
         if (c >= nchunks) continue;
-        const int64_t qpos = c * 32 + lane;
 
         // pair pass over packed items (task t, sub-chunk s): lane (k, r) = item k, member r of sub-chunk s; the
         // competitor comes from the lane that holds it (shuffle); misses run Alg. 3 lines 10-12 cooperatively
         auto pair_pass = [&](int base, int cnt) {
             const int k8 = lane >> 2, r = lane & 3;
-            const uint32_t it = iq[base + min(k8, cnt - 1)];
+            const uint32_t it = lds_u32(iq_s + 4u * (base + min(k8, cnt - 1)));
             const int t = (int)(it >> 3), src = (int)((it & 7u) << 2) + r;
             uint32_t qq[G::CW], x[G::CW];
 #pragma unroll
             for (int k = 0; k < G::CW; k++) qq[k] = __shfl_sync(0xffffffffu, q[k], src);
-            load_row<G::CW>(pV + t * CWV, x);
+            load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
 #pragma unroll
             for (int k = 0; k < G::CW; k++) x[k] -= qq[k];  // guard <=> code(q) <= code(p)
             const uint32_t M = gather_mask<G::NG>(x);
-            const uint32_t wd = state[t * C::PS + (M >> 5)];
+            const uint32_t wd = lds_u32(st_s + 4u * (t * C::PS + (M >> 5)));
             const bool miss = k8 < cnt && !(__funnelshift_r(wd, wd, M) & 1u);
             if (!__any_sync(0xffffffffu, miss)) return;  // Λ4 for every lane
             uint32_t L = 0, S = 0;
@@ -360,19 +424,19 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         uint32_t nsub32 = 0, nitem32 = 0;
         auto sub_pass = [&](int base, int cnt) {
             const int u = lane >> 3;
-            const int t = wq[base + min(u, cnt - 1)];
+            const int t = (int)lds_u32(wq_s + 4u * (base + min(u, cnt - 1)));
             uint32_t x[G::CW];
-            load_row<G::CW>(pV + t * CWV, x);
+            load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
 #pragma unroll
             for (int k = 0; k < G::CW; k++) x[k] -= sc[k];  // guard <=> sub-corner <= p
             const uint32_t Ms = gather_mask<G::NG>(x);
-            const uint32_t ws = state[t * C::PS + (Ms >> 5)];
+            const uint32_t ws = lds_u32(st_s + 4u * (t * C::PS + (Ms >> 5)));
             const bool open = u < cnt && !(__funnelshift_r(ws, ws, Ms) & 1u);
             const uint32_t ob = __ballot_sync(0xffffffffu, open);
             nsub32 += 8 * cnt;
             if (!ob) return;
             nitem32 += __popc(ob);
-            if (open) iq[iqn + __popc(ob & ((1u << lane) - 1u))] = ((uint32_t)t << 3) | (uint32_t)(lane & 7);
+            if (open) sts_u32(iq_s + 4u * (iqn + __popc(ob & ((1u << lane) - 1u))), ((uint32_t)t << 3) | (uint32_t)(lane & 7));
             iqn += __popc(ob);
             __syncwarp();
             while (iqn >= 8) {
@@ -382,19 +446,12 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             __syncwarp();
         };
 
-        // box pass; the tasks whose chunk must be opened are pooled across task groups in a per-warp queue
+        // box pass; the tasks whose chunk must be opened are pooled across task groups in a per-warp queue.
+        // Two task groups per iteration: their mask chains and probes are independent (ILP).
         int qn = 0;
-        for (int g = 0; g < ngroups; g++) {
-            const int tt = min(g * 32 + lane, nt - 1);
-            uint32_t le[G::CW];
-#pragma unroll
-            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
-            const uint32_t Mb = gather_mask<G::NG>(le);
-            const uint32_t wb = state[tt * C::PS + (Mb >> 5)];
-            const bool open = g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u);
-            const uint32_t todo = __ballot_sync(0xffffffffu, open);
-            if (todo == 0) continue;
-            if (open) wq[qn + __popc(todo & ((1u << lane) - 1u))] = g * 32 + lane;
+        auto enqueue = [&](uint32_t todo, int g) {
+            if (todo == 0) return;
+            if ((todo >> lane) & 1u) sts_u32(wq_s + 4u * (qn + __popc(todo & ((1u << lane) - 1u))), (uint32_t)(g * 32 + lane));
             qn += __popc(todo);
             __syncwarp();
             while (qn >= 4) {
@@ -402,6 +459,34 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
                 sub_pass(qn, 4);
             }
             __syncwarp();
+        };
+        auto box_test = [&](int tt, uint32_t &Mb) {
+            uint32_t le[G::CW];
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
+            Mb = gather_mask<G::NG>(le);
+        };
+        int g = 0;
+        for (; g + 1 < ngroups; g += 2) {
+            const int tt0 = g * 32 + lane, tt1 = min((g + 1) * 32 + lane, nt - 1);
+            uint32_t Mb0, Mb1;
+            box_test(tt0, Mb0);
+            box_test(tt1, Mb1);
+            const uint32_t wb0 = lds_u32(st_s + 4u * (tt0 * C::PS + (Mb0 >> 5)));
+            const uint32_t wb1 = lds_u32(st_s + 4u * (tt1 * C::PS + (Mb1 >> 5)));
+            const bool open0 = !(__funnelshift_r(wb0, wb0, Mb0) & 1u);
+            const bool open1 = (g + 1) * 32 + lane < nt && !(__funnelshift_r(wb1, wb1, Mb1) & 1u);
+            const uint32_t todo0 = __ballot_sync(0xffffffffu, open0), todo1 = __ballot_sync(0xffffffffu, open1);
+            if ((todo0 | todo1) == 0) continue;
+            enqueue(todo0, g);
+            enqueue(todo1, g + 1);
+        }
+        if (g < ngroups) {  // odd group count (always the case at d >= 15: one group per CTA)
+            const int tt = min(g * 32 + lane, nt - 1);
+            uint32_t Mb;
+            box_test(tt, Mb);
+            const uint32_t wb = lds_u32(st_s + 4u * (tt * C::PS + (Mb >> 5)));
+            enqueue(__ballot_sync(0xffffffffu, g * 32 + lane < nt && !(__funnelshift_r(wb, wb, Mb) & 1u)), g);
         }
         if (qn > 0) sub_pass(0, qn);
         if (iqn > 0) pair_pass(0, iqn);
@@ -422,38 +507,262 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         }
     }
     consumer_sync(kWarps * 32);
-    // B_{p notin S} -> membership row (its complement; bit 0, the empty subspace, is never a member)
-    for (int t = warp; t < nt; t += kWarps) {
-        const int64_t jt = j0 + t;
-        const uint32_t *st = state + t * C::PS;
-        uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-        const uint32_t *trg = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-        for (int w = lane; w < G::WB; w += 32) {
-            uint32_t v;
-            if (MODE == kModeDims) {  // p dominated in delta <=> delta in D_i for some i in delta
-                v = 0;
+    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32);
+}
+
+
+// CW words (CW even) from an 8-byte aligned shared address: the rows of a chunk record.
+template <int CW>
+__device__ __forceinline__ void load_row2_s(uint32_t a, uint32_t *w) {
 #pragma unroll
-                for (int i = 0; i < D; i++) v |= st[(1 + i) * G::WB + w] & dim_in_word(i, w);
-            } else {
-                v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+    for (int k = 0; k < CW; k += 2) asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(w[k]), "=r"(w[k + 1]) : "r"(a + 4u * k));
+}
+
+// ------------------------------------------------------------------------------------------------------
+// Design O ("task owner", d <= 15): every consumer warp owns one group of 32 tasks (codes in registers, one
+// task per lane) and a share of the chunks of every tile (wpg = 16 / groups warps per group split the 16
+// chunks).  The chunk-corner test is then lane-parallel over tasks against a broadcast corner: no task-code
+// reloads, no per-group loop.  Opened (task, chunk) items are queued and run through the same sub-chunk and
+// pair passes as design A, reading the chunk's sub-corners and competitors from the ring stage, which the
+// warp holds until it has finished the tile.  Needs 32 tasks' state in shared memory (d <= 15).
+template <int D, int MODE>
+__global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
+    const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
+    const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
+    int64_t j_end, uint32_t inexact, int ngrp, int max_level, uint32_t *__restrict__ rows32,
+    uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters) {
+    using G = Geo<D>;
+    using C = GeoK3<D, MODE>;
+    constexpr bool TIES = MODE == kModeSmemTie;
+    constexpr int CWV = C::CWV, REC = C::REC;
+    extern __shared__ __align__(128) uint32_t smem[];
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
+    const int tpc = ngrp * 32;
+    uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits
+    uint32_t *state = pV + tpc * CWV;          // [tpc][PS]
+    uint32_t *zm = state + tpc * C::PS;        // [tpc] Z_p (kModeDims)
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t *q1 = zm + tpc + warp * C::QW;    // opened (task, chunk) items (<= 3 + 32)
+    uint32_t *q2 = q1 + 40;                    // opened (task, chunk, sub-chunk) items (<= 7 + 32)
+    const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
+    const int nt = (int)min((int64_t)tpc, j_end - j0);
+    const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
+
+    if (threadIdx.x == 0) ring.init(kWarps);
+    for (int i = threadIdx.x; i < tpc * G::CW; i += blockDim.x) {
+        const int t = i / G::CW, k = i % G::CW;
+        uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
+        if (2 * k >= D) w &= 0xffff0000u;  // padding dimensions: p = 0 never passes q <= p (q pad = 1)
+        if (2 * k + 1 >= D) w &= 0x0000ffffu;
+        pV[t * CWV + k] = w | kGuard;
+    }
+    if (MODE == kModeDims) {
+        for (int t = threadIdx.x; t < tpc; t += blockDim.x) {
+            uint32_t z = 0;
+            if (t < nt)
+                for (int i = 0; i < D; i++)
+                    if (p_ord[(j0 + t) * D + i] == minord[i]) z |= 1u << i;
+            zm[t] = z;
+        }
+        __syncthreads();
+        for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) {
+            const int t = i / C::PS, w = i % C::PS;
+            const uint32_t z = zm[t], zh = z >> 5;
+            state[i] = w < G::WB && (w & ~zh) == 0 ? sub5(z & 31u) : 0u;
+        }
+    } else {
+        for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) state[i] = (i % C::PS) == 0 ? 1u : 0u;
+    }
+    __syncthreads();
+    if (warp == kWarps) {  // producer warp: one elected lane streams chunk tiles with TMA
+        if (lane == 0)
+            for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
+        return;
+    }
+    const uint32_t st_s = smem_addr(state), pV_s = smem_addr(pV), q1_s = smem_addr(q1), q2_s = smem_addr(q2);
+    const uint32_t ring_s = smem_addr(smem + 4 * kStages);
+    const int wpg = kWarps / ngrp, grp = warp / wpg, wsub = warp % wpg;
+    const int town = grp * 32 + lane;                         // this lane's task
+    const uint32_t valid = __ballot_sync(0xffffffffu, town < nt);
+    uint32_t p[G::CW];
+    load_row_s<G::CW>(pV_s + 4u * (town * CWV), p);
+    const uint32_t st_own = st_s + 4u * (town * C::PS);
+    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0;
+    for (int64_t tile = 0; tile < ntiles; tile++) {
+        ring.wait(tile);
+        const uint32_t stg_s = ring_s + 4u * (uint32_t)(tile % kStages) * (uint32_t)C::TW;
+
+        // pair pass over 8 queued (task, chunk, sub-chunk) items: lane (k, r) = item k, member r
+        auto pair_pass = [&](int base, int cnt) {
+            const int k8 = lane >> 2, r = lane & 3;
+            const uint32_t it = lds_u32(q2_s + 4u * (base + min(k8, cnt - 1)));
+            const int t = (int)(it >> 7), cl = (int)((it >> 3) & 15u), sidx = (int)(it & 7u);
+            const int m = sidx * kSubSize + r;                       // member of the chunk
+            uint32_t qq[G::CW], x[G::CW], ph[G::CW];
+            load_row2_s<G::CW>(stg_s + 4u * (cl * REC + m * G::CW), qq);
+            load_row_s<G::CW>(pV_s + 4u * (t * CWV), ph);
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) x[k] = ph[k] - qq[k];  // guard <=> code(q) <= code(p)
+            const uint32_t M = gather_mask<G::NG>(x);
+            const uint32_t wd = lds_u32(st_s + 4u * (t * C::PS + (M >> 5)));
+            const bool miss = k8 < cnt && !(__funnelshift_r(wd, wd, M) & 1u);
+            if (!__any_sync(0xffffffffu, miss)) return;  // Λ4 for every lane
+            uint32_t L = 0, S = 0;
+            if (miss) {
+                n_miss++;
+                const int64_t qpos = (tile * kWarps + cl) * 32 + m;
+                exact_masks<D>(ph, qq, M, inexact, q_ord + qpos * D, p_ord + (j0 + t) * D, L, S);
+                const uint32_t *st = state + t * C::PS;
+                if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
             }
-            const uint32_t lvl = max_level > 0 ? level_pattern(max_level - __popc(w)) : 0xffffffffu;
-            uint32_t row = ~v & G::kRowMask & lvl;
-            if (w == 0) row &= ~1u;
-            out[w * 32] = row;
-            if (ext_rows32) {
-                uint32_t er = ~st[w] & G::kRowMask & lvl;
-                if (w == 0) er &= ~1u;
-                ext_rows32[(jt >> 5) * (G::WB * 32) + w * 32 + (jt & 31)] = er;
+            uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
+            while (todo) {
+                const int from = __ffs(todo) - 1;
+                todo &= todo - 1;
+                const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
+                const int tb = __shfl_sync(0xffffffffu, t, from);
+                uint32_t *st = state + tb * C::PS;
+                const int64_t jt = j0 + tb;
+                uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+                expand<D, MODE>(st, tr, TIES ? 1 : 32, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
             }
+        };
+
+        // sub-chunk pass over 4 queued (task, chunk) items: lane (u, s) tests item u against sub-corner s
+        int n2 = 0;
+        auto sub_pass = [&](int base, int cnt) {
+            const int u = lane >> 3, sidx = lane & 7;
+            const uint32_t it = lds_u32(q1_s + 4u * (base + min(u, cnt - 1)));
+            const int t = (int)(it >> 4), cl = (int)(it & 15u);
+            uint32_t x[G::CW], sc[G::CW];
+            load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
+            load_row2_s<G::CW>(stg_s + 4u * (cl * REC + (33 + sidx) * G::CW), sc);
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) x[k] -= sc[k];  // guard <=> sub-corner <= p
+            const uint32_t Ms = gather_mask<G::NG>(x);
+            const uint32_t ws = lds_u32(st_s + 4u * (t * C::PS + (Ms >> 5)));
+            const bool open = u < cnt && !(__funnelshift_r(ws, ws, Ms) & 1u);
+            const uint32_t ob = __ballot_sync(0xffffffffu, open);
+            n_sub += 8 * cnt;
+            if (!ob) return;
+            n_pair += 4 * __popc(ob);
+            if (open) sts_u32(q2_s + 4u * (n2 + __popc(ob & ((1u << lane) - 1u))), ((uint32_t)t << 7) | ((uint32_t)cl << 3) | (uint32_t)sidx);
+            n2 += __popc(ob);
+            __syncwarp();
+            while (n2 >= 8) {
+                n2 -= 8;
+                pair_pass(n2, 8);
+            }
+            __syncwarp();
+        };
+
+        // chunk-corner (box) test: lane = task, the corner is broadcast; two chunks per iteration (ILP)
+        int n1 = 0;
+        auto enqueue = [&](uint32_t todo, int cl) {
+            if (todo == 0) return;
+            if ((todo >> lane) & 1u)
+                sts_u32(q1_s + 4u * (n1 + __popc(todo & ((1u << lane) - 1u))), ((uint32_t)town << 4) | (uint32_t)cl);
+            n1 += __popc(todo);
+            __syncwarp();
+            while (n1 >= 4) {
+                n1 -= 4;
+                sub_pass(n1, 4);
+            }
+            __syncwarp();
+        };
+        auto box_mask = [&](int cl) {
+            uint32_t mn[G::CW], le[G::CW];
+            load_row2_s<G::CW>(stg_s + 4u * (cl * REC + 32 * G::CW), mn);
+#pragma unroll
+            for (int k = 0; k < G::CW; k++) le[k] = p[k] - mn[k];  // guard <=> corner <= p
+            return gather_mask<G::NG>(le);
+        };
+        const int nch_tile = (int)min((int64_t)kWarps, nchunks - tile * kWarps);
+        const bool mine = (valid >> lane) & 1u;
+        int cl = wsub;
+        for (; cl + wpg < nch_tile; cl += 2 * wpg) {
+            const uint32_t M0 = box_mask(cl), M1 = box_mask(cl + wpg);
+            const uint32_t w0 = lds_u32(st_own + 4u * (M0 >> 5)), w1 = lds_u32(st_own + 4u * (M1 >> 5));
+            const uint32_t todo0 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w0, w0, M0) & 1u));
+            const uint32_t todo1 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w1, w1, M1) & 1u));
+            n_box += 2 * __popc(valid);
+            if ((todo0 | todo1) == 0) continue;
+            enqueue(todo0, cl);
+            enqueue(todo1, cl + wpg);
+        }
+        if (cl < nch_tile) {
+            const uint32_t M0 = box_mask(cl);
+            const uint32_t w0 = lds_u32(st_own + 4u * (M0 >> 5));
+            n_box += __popc(valid);
+            enqueue(__ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w0, w0, M0) & 1u)), cl);
+        }
+        if (n1 > 0) sub_pass(0, n1);
+        if (n2 > 0) pair_pass(0, n2);
+        // every read of the stage has completed (values consumed) before it is handed back to the producer
+        __threadfence_block();
+        __syncwarp();
+        if (lane == 0) ring.release(tile);
+    }
+    if (counters) {
+        for (int o = 16; o; o >>= 1) n_miss += __shfl_xor_sync(0xffffffffu, n_miss, o);
+        if (lane == 0) {
+            atomicAdd(&counters[2], n_box);
+            atomicAdd(&counters[3], n_pair);
+            atomicAdd(&counters[4], n_miss);
+            atomicAdd(&counters[5], n_sub);
         }
     }
+    consumer_sync(kWarps * 32);
+    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32);
+}
+
+template <int D, int MODE>
+size_t owner_smem_bytes(int ngrp) {
+    using C = GeoK3<D, MODE>;
+    const size_t tpc = (size_t)ngrp * 32;
+    return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + C::PS + 1) + kWarps * C::QW);
+}
+
+// Largest power-of-two task-group count (<= 16) whose state fits in shared memory; 0 if not even one.
+template <int D, int MODE>
+int owner_max_groups() {
+    int g = 16;
+    while (g >= 1 && owner_smem_bytes<D, MODE>(g) > (size_t)kSmemBytes) g >>= 1;
+    return g;
+}
+
+template <int D, int MODE>
+bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+    const int gmax = owner_max_groups<D, MODE>();
+    if (gmax < 1) return false;
+    const int64_t range = j_end - j_begin;
+    // groups per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
+    const int64_t want = std::max<int64_t>(1, ceil_div(ceil_div(range, c.num_sms), 32));
+    int ngrp = 1;
+    while (ngrp * 2 <= gmax && ngrp * 2 <= want) ngrp *= 2;
+    const size_t smem = owner_smem_bytes<D, MODE>(ngrp);
+    SKY_CUDA(cudaFuncSetAttribute(k3_owner_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const unsigned blocks = (unsigned)ceil_div(range, ngrp * 32);
+    k3_owner_kernel<D, MODE><<<blocks, (kWarps + 1) * 32, smem, st>>>(
+        c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
+        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp,
+        (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32, c.tie.as<uint32_t>(), ext_rows32,
+        c.counters.as<unsigned long long>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    return true;
 }
 
 template <int D, int MODE>
 void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
     using C = GeoK3<D, MODE>;
     static_assert(C::NT >= 1, "shared memory too small for one task per CTA");
+    // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
+    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  SKYCUBE_K3_DESIGN=A|O forces one.
+    const char *design = getenv("SKYCUBE_K3_DESIGN");
+    const bool want_o = design && *design ? design[0] == 'O' : MODE == kModeDims;
+    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, st)) return;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
     const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));

@@ -125,6 +125,21 @@ struct TileRing {
     }
     __device__ __forceinline__ void wait(int64_t t) const { mbar_wait(&full[t % S], (uint32_t)((t / S) & 1)); }
     __device__ __forceinline__ void release(int64_t t) const { mbar_arrive(&empty[t % S]); }
+
+    // Filtered streams: the producer fills ring slot k (the k-th streamed tile) with source tile t.
+    __device__ __forceinline__ void wait_empty(int64_t slot) const {
+        if (slot >= S) mbar_wait_sleep(&empty[slot % S], (uint32_t)(((slot / S) - 1) & 1));
+    }
+    __device__ __forceinline__ void issue2_slot(const uint32_t *a, uint32_t na, const uint32_t *b, uint32_t nb, int64_t t,
+                                                int64_t slot) const {
+        const int s = (int)(slot % S);
+        mbar_arrive_expect_tx(&full[s], (na + nb) * 4u);
+        uint32_t *dst = buf + (uint32_t)s * tile_words;
+        bulk_g2s(dst, a + t * (int64_t)na, na * 4u, &full[s]);
+        bulk_g2s(dst + na, b + t * (int64_t)nb, nb * 4u, &full[s]);
+    }
+    // completes the slot's phase without data (an end-of-stream marker stored in shared memory before it)
+    __device__ __forceinline__ void arrive_full(int64_t slot) const { mbar_arrive(&full[slot % S]); }
 };
 
 // Named barrier 1 over the consumer warps (the producer warp has left the CTA-wide barrier 0).

@@ -200,3 +200,21 @@ def test_repeat_builds_multi_tile_high_d(d):
     want = oracle.rows_b(x)
     for _ in range(6):
         assert np.array_equal(sky.skycube_build(x)["rows"], want)
+
+
+@pytest.mark.parametrize("design", ["A", "O"])
+@pytest.mark.parametrize("mode", ["0", "1", "2"])
+@pytest.mark.parametrize("case", [("A", 6000, 12, 901), ("I", 5000, 9, 902), ("A", 3000, 14, 903), ("C", 4000, 6, 904)])
+def test_k3_designs_and_modes(monkeypatch, design, mode, case):
+    """Both K3 designs (A: chunk-owner warps; O: task-owner warps, the default where 32 tasks' state fits in
+    shared memory) under every state mode, on continuous data spanning many chunk tiles with ragged tails."""
+    monkeypatch.setenv("SKYCUBE_K3_DESIGN", design)
+    monkeypatch.setenv("SKYCUBE_K3_MODE", mode)
+    dist, n, d, seed = case
+    x = datagen.generate(dist, n, d, seed)
+    want = oracle.rows_b(x)
+    r = sky.skycube_build(x)
+    bad = np.nonzero((r["rows"] != want).any(axis=1))[0]
+    assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
+    off, ids = oracle.lattice(want, d)
+    assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)

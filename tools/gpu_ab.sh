@@ -1,20 +1,18 @@
 #!/bin/bash
-# GPU-box helper: parity tests, then bench lines per config for each value of an env switch.
-#   VAR=SKYCUBE_K3_SUPER VALUES="0 1" CONFIGS="H C5" bash tools/gpu_ab.sh
+# GPU-box helper: GPU tests, then bench lines for CONFIGS under each K3 design (A, O), then (NCU=1) an ncu
+# capture of K3 at H with the default design.
 mkdir -p gpurun_out
-python -c "from paper_conf_sigmod_boghcsa17_b200 import build; build.build()" || exit 1
-if [ -z "$NO_TEST" ]; then
-  timeout 900 python -m pytest tests -m gpu -x -q ${PYTEST_K:+-k "$PYTEST_K"} > gpurun_out/pytest_gpu.log 2>&1
-  tail -3 gpurun_out/pytest_gpu.log
-fi
+python -c "from paper_conf_sigmod_boghcsa17_b200 import build; build.build()"
+timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -6 > gpurun_out/ab_tests.log
+cat gpurun_out/ab_tests.log
 for c in ${CONFIGS:-H}; do
-  for v in ${VALUES:-default}; do
-    tag=$(basename "$v")
-    if [ "$v" = default ]; then
-      timeout 600 python bench.py --steps ${STEPS:-3} --warmup 3 --config $c --no-cpu --no-e2e 2>gpurun_out/ab_${c}_$tag.err | tail -1 > gpurun_out/ab_${c}_$tag.json
-    else
-      env $VAR=$v timeout 600 python bench.py --steps ${STEPS:-3} --warmup 3 --config $c --no-cpu --no-e2e 2>gpurun_out/ab_${c}_$tag.err | tail -1 > gpurun_out/ab_${c}_$tag.json
-    fi
-    python tools/bench_summary.py gpurun_out/ab_${c}_$tag.json "$c $VAR=$v"
+  for des in ${DESIGNS:-A O}; do
+    SKYCUBE_K3_DESIGN=$des timeout 600 python bench.py --steps 3 --warmup 3 --config $c --no-e2e --no-cpu 2>/dev/null | tail -1 > gpurun_out/ab_${c}_$des.json
+    python tools/bench_summary.py gpurun_out/ab_${c}_$des.json $des
   done
 done
+if [ -n "$NCU" ]; then
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:${KERNEL:-k3_} -c 1 -f -o gpurun_out/ab_prof \
+    python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config ${NCU_CFG:-H} > gpurun_out/ab_ncu.log 2>&1
+  tail -2 gpurun_out/ab_ncu.log
+fi
