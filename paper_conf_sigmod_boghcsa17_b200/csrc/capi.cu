@@ -15,6 +15,8 @@
 struct skycube_ctx {
     sky::Ctx c;
     sky::DevBuf input, ext8, rows32, ext_rows32, membership, offsets, ids;
+    cudaStream_t side = nullptr;  // non-blocking stream for work that overlaps the main (default) stream
+    cudaEvent_t ev_ext = nullptr, ev_side = nullptr;
 };
 
 namespace {
@@ -139,7 +141,7 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
 // rows of the S+ points).  Events: ev[0] before H2D, ev[1] after H2D, ev[2] after prepare, ev[3] after
 // the prefilter, ev[4] after MDMC.
 void device_rows(skycube_ctx *x, const float *points, int64_t n, int d, int max_level, bool want_ext,
-                 cudaStream_t s, cudaEvent_t *ev) {
+                 cudaStream_t s, cudaEvent_t *ev, uint32_t *host_mem = nullptr) {
     sky::Ctx &c = x->c;
     const uint32_t W = sky::words_per_row(d);
     x->input.ensure(sizeof(float) * n * d);
@@ -157,7 +159,20 @@ void device_rows(skycube_ctx *x, const float *points, int64_t n, int d, int max_
     x->rows32.ensure(sizeof(uint32_t) * rows_words);
     if (want_ext) x->ext_rows32.ensure(sizeof(uint32_t) * rows_words);
     c.max_level = max_level;
-    sky::mdmc_run(c, 0, m, x->rows32.as<uint32_t>(), want_ext ? x->ext_rows32.as<uint32_t>() : nullptr, s);
+    if (host_mem) {
+        // zero-copy membership: the rows of points outside S+ are zeroed in the pinned host array on a side
+        // stream while K3 runs (and writes the S+ rows there itself); the caller joins x->ev_side
+        if (!x->side) {
+            SKY_CUDA(cudaStreamCreateWithFlags(&x->side, cudaStreamNonBlocking));
+            SKY_CUDA(cudaEventCreateWithFlags(&x->ev_ext, cudaEventDisableTiming));
+            SKY_CUDA(cudaEventCreateWithFlags(&x->ev_side, cudaEventDisableTiming));
+        }
+        SKY_CUDA(cudaEventRecord(x->ev_ext, s));
+        SKY_CUDA(cudaStreamWaitEvent(x->side, x->ev_ext, 0));
+        sky::membership_zero_outside(c, host_mem, x->side);
+        SKY_CUDA(cudaEventRecord(x->ev_side, x->side));
+    }
+    sky::mdmc_run(c, 0, m, x->rows32.as<uint32_t>(), want_ext ? x->ext_rows32.as<uint32_t>() : nullptr, s, host_mem);
     SKY_CUDA(cudaEventRecord(ev[4], s));
 }
 
@@ -238,10 +253,16 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
         cudaStream_t s = nullptr;
         Events evs;
         cudaEvent_t *ev = evs.e;
-        device_rows(x, points, n, d, max_level, want_ext, s, ev);
+        // membership goes to the pinned result buffer by zero-copy from K3 (unless the debug ext rows are
+        // requested: then the device transpose + copy path below)
+        r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
+        uint32_t *host_mem = want_ext ? nullptr : r.membership;
+        device_rows(x, points, n, d, max_level, want_ext, s, ev, host_mem);
         const int64_t m = c.m;
-        x->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
-        sky::compact_membership(c, x->rows32.as<uint32_t>(), x->membership.as<uint32_t>(), s);
+        if (!host_mem) {
+            x->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
+            sky::compact_membership(c, x->rows32.as<uint32_t>(), x->membership.as<uint32_t>(), s);
+        }
         int64_t total = 0;
         const bool lists = !(flags & SKYCUBE_NO_LISTS);
         if (lists) {
@@ -254,10 +275,13 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
         // device -> pinned host
         r.n_ext = m;
         r.ext_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (m > 0 ? m : 1));
-        r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
         if (m) SKY_CUDA(cudaMemcpyAsync(r.ext_ids, c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, s));
-        SKY_CUDA(cudaMemcpyAsync(r.membership, x->membership.p, sizeof(uint32_t) * (size_t)n * W,
-                                 cudaMemcpyDeviceToHost, s));
+        if (host_mem) {
+            SKY_CUDA(cudaStreamWaitEvent(s, x->ev_side, 0));
+        } else {
+            SKY_CUDA(cudaMemcpyAsync(r.membership, x->membership.p, sizeof(uint32_t) * (size_t)n * W,
+                                     cudaMemcpyDeviceToHost, s));
+        }
         if (lists) {
             r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
             r.cuboid_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (total > 0 ? total : 1));
@@ -431,6 +455,9 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
                            &ctx->membership, &ctx->offsets, &ctx->ids})
         b->release();
     c.hc.release();
+    if (ctx->side) cudaStreamDestroy(ctx->side);
+    if (ctx->ev_ext) cudaEventDestroy(ctx->ev_ext);
+    if (ctx->ev_side) cudaEventDestroy(ctx->ev_side);
     delete ctx;
 }
 

@@ -101,9 +101,13 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st);
 // k1_prefilter.cu
 void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ext_sorted, cudaStream_t st);
 // k3_mdmc.cu
-void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st);
+// host_membership (nullable): pinned host array [n][W] that also receives every S+ row by point id (zero-copy)
+void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st,
+              uint32_t *host_membership = nullptr);
 // k4_compact.cu
 void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cudaStream_t st);
+// zero rows of the points outside S+ in a (host-mapped) membership array [n][W] (zero-copy path)
+void membership_zero_outside(Ctx &c, uint32_t *membership, cudaStream_t st);
 void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
                      cudaStream_t st);
 // k5_hashcube.cu

@@ -31,7 +31,10 @@ namespace {
 
 constexpr int kWarps = 16;                   // consumer warps (+1 producer warp)
 constexpr int kTasks = kWarps * 32;          // tasks (tree positions) per CTA
-constexpr int kStages = 4;
+// ring depth: 6 stages cover the bulk-copy latency of the (filtered) tile stream; at d > 12 (CW = 8) only 4
+// fit with two CTAs per SM
+template <int CW>
+constexpr int stages_for() { return CW <= 6 ? 6 : 4; }
 
 template <int CW>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
@@ -42,6 +45,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
     constexpr int CWS = (CW + 3) & ~3;  // tile-corner record words
     constexpr int CWV = (CW + 3) & ~3;  // 16-byte task-code stride (broadcast vector loads)
     constexpr int TW = kTileChunks * REC + CWS;
+    constexpr int kStages = stages_for<CW>();
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)TW};
@@ -84,35 +88,47 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
     }
     __syncthreads();
     if (warp == kWarps) {
-        // producer warp: one elected lane streams only the tiles whose corner is below the CTA's upper
-        // corner U (per-dimension maximum code of its tasks) -- no other tile can hold a dominator of any
-        // task here -- and publishes each streamed tile's index with its ring slot; -1 ends the stream
-        if (lane == 0) {
-            uint32_t um[CW];
+        // producer warp: streams only the tiles whose corner is below the CTA's upper corner U (per-dimension
+        // maximum code of its tasks) -- no other tile can hold a dominator of any task here -- and publishes
+        // each streamed tile's index with its ring slot; -1 ends the stream.  The 32 lanes test 32 tile
+        // corners at a time (independent loads); lane 0 issues the bulk copies in order.
+        uint32_t um[CW];
 #pragma unroll
-            for (int k = 0; k < CW; k++) um[k] = 0;
+        for (int k = 0; k < CW; k++) um[k] = 0;
 #pragma unroll
-            for (int w = 0; w < kWarps; w++) {
+        for (int w = 0; w < kWarps; w++) {
 #pragma unroll
-                for (int k = 0; k < CW; k++) {
-                    const uint32_t u = ucorner[w * CW + k];
-                    um[k] = max(um[k] & 0xffffu, u & 0xffffu) | (max(um[k] >> 16, u >> 16) << 16);
-                }
+            for (int k = 0; k < CW; k++) {
+                const uint32_t u = ucorner[w * CW + k];
+                um[k] = max(um[k] & 0xffffu, u & 0xffffu) | (max(um[k] >> 16, u >> 16) << 16);
             }
+        }
 #pragma unroll
-            for (int k = 0; k < CW; k++) um[k] = (um[k] | kGuard) - csub[k];
-            int64_t slot = 0;
-            for (int64_t t = 0; t < ntiles; t++) {
+        for (int k = 0; k < CW; k++) um[k] = (um[k] | kGuard) - csub[k];
+        int64_t slot = 0;
+        for (int64_t t0 = 0; t0 < ntiles; t0 += 32) {
+            const int64_t t = t0 + lane;
+            bool pass = false;
+            if (t < ntiles) {
                 const uint32_t *sc = supers + t * CWS;
                 uint32_t acc = 0xffffffffu;
 #pragma unroll
                 for (int k = 0; k < CW; k++) acc &= um[k] - __ldg(sc + k);
-                if ((acc & kGuard) != kGuard) continue;
-                ring.wait_empty(slot);
-                tile_idx[slot % kStages] = (int32_t)t;
-                ring.issue2_slot(chunks, kTileChunks * REC, supers, CWS, t, slot);
+                pass = (acc & kGuard) == kGuard;
+            }
+            uint32_t m = __ballot_sync(0xffffffffu, pass);
+            while (m) {
+                const int b = __ffs(m) - 1;
+                m &= m - 1;
+                if (lane == 0) {
+                    ring.wait_empty(slot);
+                    tile_idx[slot % kStages] = (int32_t)(t0 + b);
+                    ring.issue2_slot(chunks, kTileChunks * REC, supers, CWS, t0 + b, slot);
+                }
                 slot++;
             }
+        }
+        if (lane == 0) {
             ring.wait_empty(slot);
             tile_idx[slot % kStages] = -1;
             ring.arrive_full(slot);
@@ -198,6 +214,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
 
 template <int CW>
 void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uint8_t *ext, cudaStream_t st) {
+    constexpr int kStages = stages_for<CW>();
     const size_t smem = sizeof(uint32_t) * (4 * kStages + (size_t)kStages * (kTileChunks * 33 * CW + ((CW + 3) & ~3)) +
                                             (size_t)kTasks * ((CW + 3) & ~3) + kStages + (size_t)kWarps * CW);
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

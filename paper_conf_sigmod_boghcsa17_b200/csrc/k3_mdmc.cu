@@ -270,7 +270,8 @@ __device__ __forceinline__ void load_row_s(uint32_t a, uint32_t *w) {
 template <int D, int MODE>
 __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, int nt, int warp, int lane, int max_level,
                                            uint32_t *__restrict__ rows32, const uint32_t *__restrict__ tie32,
-                                           uint32_t *__restrict__ ext_rows32) {
+                                           uint32_t *__restrict__ ext_rows32, uint32_t *__restrict__ host_mem,
+                                           const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
     constexpr bool TIES = MODE == kModeSmemTie;
@@ -279,6 +280,9 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
         const uint32_t *st = state + t * C::PS;
         uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
         const uint32_t *trg = tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
+        // zero-copy: the row also goes straight to the caller's pinned host membership array (by point id),
+        // so its PCIe transfer overlaps the rest of the kernel instead of following the whole build
+        uint32_t *hrow = host_mem ? host_mem + (int64_t)ext_ids[jt] * G::WB : nullptr;
         for (int w = lane; w < G::WB; w += 32) {
             uint32_t v;
             if (MODE == kModeDims) {  // p dominated in delta <=> delta in D_i for some i in delta
@@ -292,6 +296,7 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
             uint32_t row = ~v & G::kRowMask & lvl;
             if (w == 0) row &= ~1u;
             out[w * 32] = row;
+            if (hrow) hrow[w] = row;
             if (ext_rows32) {
                 uint32_t er = ~st[w] & G::kRowMask & lvl;
                 if (w == 0) er &= ~1u;
@@ -306,7 +311,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
     int64_t j_end, uint32_t inexact, int tpc, int max_level, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
-    uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters) {
+    uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters, uint32_t *__restrict__ host_mem,
+    const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
     constexpr bool TIES = MODE == kModeSmemTie;
@@ -507,7 +513,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         }
     }
     consumer_sync(kWarps * 32);
-    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32);
+    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
 }
 
 
@@ -530,7 +536,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
     int64_t j_end, uint32_t inexact, int ngrp, int max_level, uint32_t *__restrict__ rows32,
-    uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters) {
+    uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters,
+    uint32_t *__restrict__ host_mem, const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
     constexpr bool TIES = MODE == kModeSmemTie;
@@ -714,7 +721,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         }
     }
     consumer_sync(kWarps * 32);
-    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32);
+    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
 }
 
 template <int D, int MODE>
@@ -733,7 +740,8 @@ int owner_max_groups() {
 }
 
 template <int D, int MODE>
-bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
+                  cudaStream_t st) {
     const int gmax = owner_max_groups<D, MODE>();
     if (gmax < 1) return false;
     const int64_t range = j_end - j_begin;
@@ -748,21 +756,22 @@ bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
         c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32, c.tie.as<uint32_t>(), ext_rows32,
-        c.counters.as<unsigned long long>());
+        c.counters.as<unsigned long long>(), host_mem, c.ext_ids.as<int32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     return true;
 }
 
 template <int D, int MODE>
-void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
+              cudaStream_t st) {
     using C = GeoK3<D, MODE>;
     static_assert(C::NT >= 1, "shared memory too small for one task per CTA");
     // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
     // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  SKYCUBE_K3_DESIGN=A|O forces one.
     const char *design = getenv("SKYCUBE_K3_DESIGN");
     const bool want_o = design && *design ? design[0] == 'O' : MODE == kModeDims;
-    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, st)) return;
+    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
     const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
@@ -773,7 +782,7 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
         c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32,
-        c.tie.as<uint32_t>(), ext_rows32, c.counters.as<unsigned long long>());
+        c.tie.as<uint32_t>(), ext_rows32, c.counters.as<unsigned long long>(), host_mem, c.ext_ids.as<int32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
@@ -783,7 +792,8 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
 // data at d > 10: ties are rare and go to a global row (kModeGlobalTie).  SKYCUBE_K3_MODE=0|1|2 forces a
 // mode (parity tests of every mode on the same inputs).
 template <int D>
-void launch(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, cudaStream_t st) {
+void launch(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
+            cudaStream_t st) {
     const bool all_exact = c.exact_mask == ((1u << D) - 1u);
     const char *m = getenv("SKYCUBE_K3_MODE");
     int mode = (D <= 10 || all_exact) ? (D <= 12 && !ext_rows32 ? kModeDims : kModeSmemTie) : kModeGlobalTie;
@@ -792,17 +802,18 @@ void launch(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *
         if (mode == kModeDims && (D > 12 || ext_rows32)) mode = kModeSmemTie;
     }
     if (mode == kModeDims) {
-        if constexpr (D <= 12) launch_t<D, kModeDims>(c, j_begin, j_end, rows32, ext_rows32, st);
+        if constexpr (D <= 12) launch_t<D, kModeDims>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
     } else if (mode == kModeSmemTie) {
-        launch_t<D, kModeSmemTie>(c, j_begin, j_end, rows32, ext_rows32, st);
+        launch_t<D, kModeSmemTie>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
     } else {
-        launch_t<D, kModeGlobalTie>(c, j_begin, j_end, rows32, ext_rows32, st);
+        launch_t<D, kModeGlobalTie>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
     }
 }
 
 }  // namespace
 
-void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st) {
+void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32_t *d_ext_rows32, cudaStream_t st,
+              uint32_t *host_membership) {
     if (!c.ext_ready) throw Error{1, "skycube_dev_mdmc before skycube_dev_set_ext"};
     if (j_begin < 0 || j_end > c.m || (j_begin & 31)) throw Error{1, "bad MDMC task range"};
     if (j_end <= j_begin) return;
@@ -811,7 +822,7 @@ void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32
     c.tie.ensure(sizeof(uint32_t) * grp_words * (size_t)ceil_div(c.m, 32));
     SKY_CUDA(cudaMemsetAsync(c.tie.as<uint32_t>() + g0 * grp_words, 0, sizeof(uint32_t) * grp_words * (g1 - g0), st));
     switch (c.d) {
-#define SKY_K3(DD) case DD: launch<DD>(c, j_begin, j_end, d_rows32, d_ext_rows32, st); break;
+#define SKY_K3(DD) case DD: launch<DD>(c, j_begin, j_end, d_rows32, d_ext_rows32, host_membership, st); break;
         SKY_K3(1) SKY_K3(2) SKY_K3(3) SKY_K3(4) SKY_K3(5) SKY_K3(6) SKY_K3(7) SKY_K3(8)
         SKY_K3(9) SKY_K3(10) SKY_K3(11) SKY_K3(12) SKY_K3(13) SKY_K3(14) SKY_K3(15) SKY_K3(16)
 #undef SKY_K3

@@ -91,3 +91,61 @@ def test_c2_full_oracle(engine):
     offs, ids = oracle.lattice(want, x.shape[1])
     assert np.array_equal(out["offsets"].cpu().numpy(), offs)
     assert np.array_equal(out["ids"].cpu().numpy(), ids)
+
+
+@pytest.mark.parametrize("name", ["C3A", "C5", "H"])
+def test_full_size_hashcube_sampled(engine, name):
+    """HashCube (K5, w = 32) at full size through the bench launch path: for seeded sample points the oracle
+    row (Oracle B) fixes, word by word, the key the point must be stored under (or that it is absent); plus
+    properties: keys ascending per word, ids ascending per key, each point at most once per word, and the
+    number of stored ids = the number of not-all-dominated (point, word) pairs of the GPU's own rows."""
+    import torch
+    from oracle import hashcube as hco
+    cfg = datagen.config(name)
+    x = cfg.data()
+    n, d = x.shape
+    out = engine.build(torch.from_numpy(x).cuda(), lists=False, membership=True, hashcube_w=32)
+    torch.cuda.synchronize()
+    hc = {k: v.cpu().numpy() for k, v in out["hashcube"].items()}
+    keys = hc["keys"].view(np.uint32)
+    woff, koff, ids = hc["word_offsets"], hc["key_offsets"], hc["ids"]
+    nw = hco.n_words(d, 32)
+    assert woff.shape[0] == nw + 1 and woff[0] == 0 and woff[-1] == keys.size and koff[-1] == ids.size
+    key_word = np.repeat(np.arange(nw), np.diff(woff))
+    assert np.all((np.diff(keys.astype(np.int64)) > 0) | (np.diff(key_word) > 0)), "keys ascending per word"
+    id_key = np.repeat(np.arange(keys.size), np.diff(koff))
+    assert np.all((np.diff(ids) > 0) | (np.diff(id_key) > 0)), "ids ascending per key"
+    # where every point is stored, per word: (word, id) -> key
+    id_word = key_word[id_key]
+    pair = id_word.astype(np.int64) * n + ids
+    assert np.unique(pair).size == pair.size, "each point at most once per word"
+    ext_ids = out["ext_ids"].cpu().numpy()
+    rng = np.random.default_rng(77)
+    pids = np.unique(np.concatenate([rng.choice(ext_ids, 16, replace=False), rng.choice(n, 8, replace=False)]))
+    want = hco.hashcube(oracle.rows_b(x, pids), d, 32)  # HashCube of the sample alone (ids 0..len-1)
+    order = np.argsort(pair, kind="stable")
+    sp = pair[order]
+    for s, p in enumerate(pids):
+        for k in range(nw):
+            # oracle: key of sample point s in word k, or absent
+            lo, hi = want["word_offsets"][k], want["word_offsets"][k + 1]
+            wkey = None
+            for u in range(lo, hi):
+                if s in want["ids"][want["key_offsets"][u]:want["key_offsets"][u + 1]]:
+                    wkey = int(want["keys"][u])
+            j = np.searchsorted(sp, k * n + p)
+            found = j < sp.size and sp[j] == k * n + p
+            gkey = int(keys[id_key[order[j]]]) if found else None
+            assert gkey == wkey, f"{name}: point {p} word {k}: gpu {gkey} oracle {wkey}"
+    # stored ids == (point, word) pairs of the rows whose word is not all dominated
+    notS = ~out["membership"].cpu().numpy().view(np.uint32)
+    W = notS.shape[1]
+    stored = 0
+    for k in range(nw):
+        v = (notS[:, k].astype(np.uint64) >> np.uint64(1))
+        if k + 1 < W:
+            v |= (notS[:, k + 1].astype(np.uint64) & np.uint64(1)) << np.uint64(31)
+        valid = min(32, (1 << d) - 1 - 32 * k)
+        full = np.uint64((1 << valid) - 1)
+        stored += int(np.count_nonzero((v & full) != full))
+    assert stored == ids.size
