@@ -62,7 +62,10 @@ struct Geo {
 };
 
 constexpr int kWarps = 16;                // consumer warps = chunks per tile (+1 producer warp)
-constexpr int kStages = 4;                // TMA ring depth
+// TMA ring depth: 4 stages; at d >= 15 the 2^d-bit task state crowds shared memory (8 KB per task at d = 16),
+// and two stages buy 5 more tasks per CTA (19 -> 24)
+template <int D>
+constexpr int k3_stages() { return D >= 15 ? 2 : 4; }
 constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");
@@ -75,6 +78,7 @@ struct GeoK3 {
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
     static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
     static constexpr int TW = kWarps * REC;                              // tile words
+    static constexpr int kStages = k3_stages<D>();
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
     static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
     static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
@@ -319,6 +323,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     constexpr int CWP = C::CWP, CWV = C::CWV, REC = C::REC;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    constexpr int kStages = C::kStages;
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
     uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits (broadcast rows)
     uint32_t *pH = pV + tpc * CWV;             // [tpc][CWP] the same, odd stride (per-lane rows)
@@ -544,6 +549,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     constexpr int CWV = C::CWV, REC = C::REC;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
+    constexpr int kStages = C::kStages;
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
     const int tpc = ngrp * 32;
     uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits

@@ -51,71 +51,171 @@ __global__ void zero_outside_kernel(const uint32_t *__restrict__ ext_id_flag, in
         if (!ext_id_flag[i / W]) membership[i] = 0u;
 }
 
-// counts[delta * nchunks + c] = |S_delta restricted to chunk c|.
+// Lattice (CSR per subspace, ascending ids).  A block = NWK groups of 32 tasks ("chunk" c); per word w of
+// the rows, lane b of a warp holds (after the transpose) the task mask of subspace delta = 32w + b.
+// Counts are stored chunk-major, counts[c * NS + delta] (NS = 32 W >= 2^d), so a warp's 32 subspaces are 32
+// consecutive entries (coalesced); the offset of (delta, c) is doff[delta] + colpre[c * NS + delta], where
+// colpre is the prefix over chunks per subspace and doff the exclusive scan of the per-subspace totals.
+// UNR words per iteration keep several 128-byte row loads in flight per warp.
+constexpr int kUnr = 4;
+
 template <int NWK>
 __global__ void __launch_bounds__(NWK * 32) lattice_count_kernel(const uint32_t *__restrict__ rows32, int64_t m,
-                                                               uint32_t W, int64_t nchunks,
-                                                               uint64_t *__restrict__ counts) {
-    __shared__ uint32_t red[NWK][32];
+                                                               uint32_t W, uint64_t *__restrict__ counts) {
+    __shared__ uint32_t red[kUnr][NWK][32];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t c = blockIdx.x;
     const int64_t g = c * NWK + warp;
-    for (uint32_t w = blockIdx.y; w < W; w += gridDim.y) {
-        const uint32_t x = g * 32 + lane < m ? rows32[g * W * 32 + (int64_t)w * 32 + lane] : 0u;  // tail lanes unused
-        red[warp][lane] = __popc(transpose32(x, lane));
+    const int64_t NS = (int64_t)W * 32;
+    const bool live = g * 32 + lane < m;  // tail lanes unused
+    for (uint32_t w0 = blockIdx.y * kUnr; w0 < W; w0 += gridDim.y * kUnr) {
+        uint32_t x[kUnr];
+#pragma unroll
+        for (int u = 0; u < kUnr; u++)
+            x[u] = live && w0 + u < W ? rows32[g * W * 32 + (int64_t)(w0 + u) * 32 + lane] : 0u;
+#pragma unroll
+        for (int u = 0; u < kUnr; u++) red[u][warp][lane] = __popc(transpose32(x[u], lane));
         __syncthreads();
-        if (warp == 0) {
+        if (warp < kUnr && w0 + warp < W) {
             uint32_t s = 0;
 #pragma unroll
-            for (int k = 0; k < NWK; k++) s += red[k][lane];
-            counts[((int64_t)w * 32 + lane) * nchunks + c] = s;
+            for (int k = 0; k < NWK; k++) s += red[warp][k][lane];
+            counts[c * NS + (int64_t)(w0 + warp) * 32 + lane] = s;
         }
         __syncthreads();
     }
+}
+
+// colpre[c * NS + delta] = sum of counts of chunks < c; tot[delta] = sum over all chunks.  Thread = subspace.
+__global__ void lattice_colscan_kernel(const uint64_t *__restrict__ counts, int64_t nchunks, int64_t NS,
+                                       uint64_t *__restrict__ colpre, uint64_t *__restrict__ tot) {
+    const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (delta >= NS) return;
+    uint64_t run = 0;
+    int64_t c = 0;
+    for (; c + 4 <= nchunks; c += 4) {
+        uint64_t v[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) v[u] = counts[(c + u) * NS + delta];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            colpre[(c + u) * NS + delta] = run;
+            run += v[u];
+        }
+    }
+    for (; c < nchunks; c++) {
+        const uint64_t v = counts[c * NS + delta];
+        colpre[c * NS + delta] = run;
+        run += v;
+    }
+    tot[delta] = run;
 }
 
 // Scatter: warp = group of 32 tasks, lane = task.  After the transpose lane b holds the task mask of
 // subspace delta = 32w + b and its segment offset; the warp then writes each non-empty subspace's ids with
 // one coalesced store (the set lanes write consecutive addresses), instead of 32 lanes each appending to a
-// different list (4-byte scattered stores: 8x sector write amplification, 58 ms at d = 16).
+// different list (4-byte scattered stores: 8x sector write amplification).
 template <int NWK>
 __global__ void __launch_bounds__(NWK * 32) lattice_scatter_kernel(const uint32_t *__restrict__ rows32, int64_t m,
-                                                                 uint32_t W, int64_t nchunks,
-                                                                 const uint64_t *__restrict__ base,
+                                                                 uint32_t W, const uint64_t *__restrict__ colpre,
+                                                                 const uint64_t *__restrict__ doff,
                                                                  const int32_t *__restrict__ ext_ids,
                                                                  int32_t *__restrict__ ids) {
-    __shared__ uint32_t red[NWK][32];
+    __shared__ uint32_t red[kUnr][NWK][32];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t c = blockIdx.x;
     const int64_t g = c * NWK + warp;
+    const int64_t NS = (int64_t)W * 32;
     const int64_t j = g * 32 + lane;
-    const int32_t my_id = j < m ? ext_ids[j] : 0;
+    const bool live = j < m;
+    const int32_t my_id = live ? ext_ids[j] : 0;
     const uint32_t lt = (1u << lane) - 1u;
-    for (uint32_t w = blockIdx.y; w < W; w += gridDim.y) {
-        const uint32_t x = j < m ? rows32[g * W * 32 + (int64_t)w * 32 + lane] : 0u;  // tail lanes unused
-        const uint32_t mask = transpose32(x, lane);  // lane b: tasks of the group in subspace 32w + b
-        red[warp][lane] = __popc(mask);
+    for (uint32_t w0 = blockIdx.y * kUnr; w0 < W; w0 += gridDim.y * kUnr) {
+        uint32_t mask[kUnr];
+        uint64_t off[kUnr];
+#pragma unroll
+        for (int u = 0; u < kUnr; u++) {
+            const uint32_t x = live && w0 + u < W ? rows32[g * W * 32 + (int64_t)(w0 + u) * 32 + lane] : 0u;
+            mask[u] = transpose32(x, lane);  // lane b: tasks of the group in subspace 32(w0+u) + b
+            red[u][warp][lane] = __popc(mask[u]);
+            const int64_t delta = (int64_t)(w0 + u) * 32 + lane;
+            off[u] = w0 + u < W ? doff[delta] + colpre[c * NS + delta] : 0;
+        }
         __syncthreads();
-        uint64_t off = base[((int64_t)w * 32 + lane) * nchunks + c];
-        for (int k = 0; k < warp; k++) off += red[k][lane];
-        uint32_t nz = __ballot_sync(0xffffffffu, mask != 0u);
-        while (nz) {
-            const int b = __ffs(nz) - 1;
-            nz &= nz - 1;
-            const uint32_t mb = __shfl_sync(0xffffffffu, mask, b);
-            const uint64_t ob = __shfl_sync(0xffffffffu, off, b);
-            if ((mb >> lane) & 1u) ids[ob + __popc(mb & lt)] = my_id;
+#pragma unroll
+        for (int u = 0; u < kUnr; u++) {
+            for (int k = 0; k < warp; k++) off[u] += red[u][k][lane];
+            uint32_t nz = __ballot_sync(0xffffffffu, mask[u] != 0u);
+            while (nz) {
+                const int b = __ffs(nz) - 1;
+                nz &= nz - 1;
+                const uint32_t mb = __shfl_sync(0xffffffffu, mask[u], b);
+                const uint64_t ob = __shfl_sync(0xffffffffu, off[u], b);
+                if ((mb >> lane) & 1u) ids[ob + __popc(mb & lt)] = my_id;
+            }
         }
         __syncthreads();
     }
 }
 
-__global__ void lattice_offsets_kernel(const uint64_t *__restrict__ base, const uint64_t *__restrict__ counts,
-                                       int64_t nchunks, int64_t nsub, int64_t nentries, int64_t *__restrict__ offsets) {
+// Scatter for large subspace counts (d > 12: every (subspace, group) segment holds only a few ids, so the
+// per-group scatter above issues one store per ~4 ids).  A block = 32 groups (1024 tasks); per word w each
+// warp transposes its group's word into shared memory, then warp b takes subspace delta = 32w + b with
+// lane = group: a warp prefix sum of the 32 group counts places the whole 1024-task segment of delta, and
+// lane-parallel stores write it (one store instruction per ~32 x 4 ids).
+__global__ void __launch_bounds__(1024) lattice_scatter32_kernel(const uint32_t *__restrict__ rows32, int64_t m,
+                                                               uint32_t W, const uint64_t *__restrict__ colpre,
+                                                               const uint64_t *__restrict__ doff,
+                                                               const int32_t *__restrict__ ext_ids,
+                                                               int32_t *__restrict__ ids) {
+    __shared__ uint32_t M[32][33];  // [group][subspace bit]
+    __shared__ int32_t sid[1024];
+    extern __shared__ int32_t stage[];  // [32 warps][1024]: the warp's subspace segment, compacted
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t c = blockIdx.x;
+    const int64_t g = c * 32 + warp;
+    const int64_t NS = (int64_t)W * 32;
+    const int64_t j = g * 32 + lane;
+    int32_t *seg = stage + warp * 1024;
+    sid[threadIdx.x] = j < m ? ext_ids[j] : 0;
+    const uint32_t *rowp = rows32 + g * W * 32 + lane;
+    uint32_t x_next = j < m && blockIdx.y < W ? rowp[(int64_t)blockIdx.y * 32] : 0u;
+    for (uint32_t w = blockIdx.y; w < W; w += gridDim.y) {
+        const uint32_t x = x_next;  // this word was loaded during the previous iteration (latency hidden)
+        const uint32_t wn = w + gridDim.y;
+        x_next = j < m && wn < W ? rowp[(int64_t)wn * 32] : 0u;
+        M[warp][lane] = transpose32(x, lane);  // lane b: tasks of group `warp` in subspace 32w + b
+        __syncthreads();
+        const uint32_t mg = M[lane][warp];     // tasks of group `lane` in subspace 32w + warp
+        const uint32_t cnt = __popc(mg);
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        // compact this subspace's ids of the 1024 tasks into the warp's stage (ascending: group, then bit) ...
+        uint32_t mm = mg, o = incl - cnt;
+        while (mm) {
+            const int b = __ffs(mm) - 1;
+            mm &= mm - 1;
+            seg[o++] = sid[lane * 32 + b];
+        }
+        __syncwarp();
+        // ... and write the segment with full-line coalesced stores
+        const int64_t delta = (int64_t)w * 32 + warp;
+        int32_t *dst = ids + doff[delta] + colpre[c * NS + delta];
+        for (uint32_t i = lane; i < total; i += 32) dst[i] = seg[i];
+        __syncthreads();
+    }
+}
+
+__global__ void lattice_offsets_kernel(const uint64_t *__restrict__ doff, const uint64_t *__restrict__ tot,
+                                       int64_t nsub, int64_t *__restrict__ offsets) {
     const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (delta > nsub) return;
-    if (delta < nsub) offsets[delta] = (int64_t)base[delta * nchunks];
-    else offsets[delta] = (int64_t)(base[nentries - 1] + counts[nentries - 1]);
+    offsets[delta] = delta < nsub ? (int64_t)doff[delta] : (int64_t)(doff[nsub - 1] + tot[nsub - 1]);
 }
 
 }  // namespace
@@ -146,42 +246,50 @@ void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *
     const bool big = c.d > 12;
     const int nwk = big ? 32 : 8;
     const int64_t nchunks = ceil_div(ngroups > 0 ? ngroups : 1, nwk);
-    const int64_t nentries = (int64_t)c.W * 32 * nchunks;  // >= nsub * nchunks
-    const unsigned gy = (unsigned)std::min<int64_t>(c.W, big ? 64 : 16);
+    const int64_t NS = (int64_t)c.W * 32;  // >= nsub
+    const int64_t nentries = NS * nchunks;
+    const unsigned gy = (unsigned)std::min<int64_t>(ceil_div(c.W, kUnr), big ? 16 : 4);
     dim3 grid((unsigned)nchunks, gy);
+    c.lat_counts.ensure(sizeof(uint64_t) * (2 * (size_t)nentries + 2 * (size_t)NS));
+    uint64_t *counts = c.lat_counts.as<uint64_t>();
+    uint64_t *colpre = counts + nentries;
+    uint64_t *tot = colpre + nentries;
+    uint64_t *doff = tot + NS;
     if (ids == nullptr) {
-        c.lat_counts.ensure(sizeof(uint64_t) * 2 * (size_t)nentries);
-        c.scan64_tmp.ensure(scan_tmp_bytes(nentries));
-        uint64_t *counts = c.lat_counts.as<uint64_t>();
-        uint64_t *base = counts + nentries;
+        c.scan64_tmp.ensure(scan_tmp_bytes(NS));
         if (c.m == 0) {
-            SKY_CUDA(cudaMemsetAsync(counts, 0, sizeof(uint64_t) * 2 * (size_t)nentries, st));
-        } else if (big) {
-            lattice_count_kernel<32><<<grid, 32 * 32, 0, st>>>(rows32, c.m, c.W, nchunks, counts);
+            SKY_CUDA(cudaMemsetAsync(counts, 0, sizeof(uint64_t) * (size_t)nentries, st));
         } else {
-            lattice_count_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, nchunks, counts);
-        }
-        if (c.m) {
+            if (big)
+                lattice_count_kernel<32><<<grid, 32 * 32, 0, st>>>(rows32, c.m, c.W, counts);
+            else
+                lattice_count_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, counts);
             c.L.count++;
             SKY_LAUNCH_CHECK();
         }
-        exclusive_scan_u64(counts, base, nentries, c.scan64_tmp.p, st, c.L);
-        lattice_offsets_kernel<<<(unsigned)ceil_div(nsub + 1, 256), 256, 0, st>>>(base, counts, nchunks, nsub, nentries,
-                                                                                 offsets);
+        lattice_colscan_kernel<<<(unsigned)ceil_div(NS, 128), 128, 0, st>>>(counts, nchunks, NS, colpre, tot);
         c.L.count++;
         SKY_LAUNCH_CHECK();
-        int64_t tot = 0;
-        SKY_CUDA(cudaMemcpyAsync(&tot, offsets + nsub, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        exclusive_scan_u64(tot, doff, NS, c.scan64_tmp.p, st, c.L);
+        lattice_offsets_kernel<<<(unsigned)ceil_div(nsub + 1, 256), 256, 0, st>>>(doff, tot, nsub, offsets);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+        int64_t tot_ids = 0;
+        SKY_CUDA(cudaMemcpyAsync(&tot_ids, offsets + nsub, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
         SKY_CUDA(cudaStreamSynchronize(st));
-        *total_ids = tot;
+        *total_ids = tot_ids;
         return;
     }
     if (c.m == 0) return;
-    const uint64_t *base = c.lat_counts.as<uint64_t>() + nentries;
     if (big)
-        lattice_scatter_kernel<32><<<grid, 32 * 32, 0, st>>>(rows32, c.m, c.W, nchunks, base, c.ext_ids.as<int32_t>(), ids);
+    {
+        const int smem = 32 * 1024 * (int)sizeof(int32_t);
+        SKY_CUDA(cudaFuncSetAttribute(lattice_scatter32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        lattice_scatter32_kernel<<<dim3((unsigned)nchunks, (unsigned)std::min<int64_t>(c.W, 64)), 1024, smem, st>>>(
+            rows32, c.m, c.W, colpre, doff, c.ext_ids.as<int32_t>(), ids);
+    }
     else
-        lattice_scatter_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, nchunks, base, c.ext_ids.as<int32_t>(), ids);
+        lattice_scatter_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, colpre, doff, c.ext_ids.as<int32_t>(), ids);
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }

@@ -58,10 +58,21 @@ def chunk_words(m: int, d: int, world: int) -> int:
 
 
 # ------------------------------------------------------------------ collectives (NCCL or gloo)
+def _staged(t: torch.Tensor, group) -> bool:
+    """gloo does not run every collective on CUDA tensors: stage through host memory there (used by the
+    single-GPU multi-rank tests; NCCL never stages)."""
+    return t.is_cuda and dist.get_backend(group) == "gloo"
+
+
 def exchange_ext(ext8: torch.Tensor, group=None):
     """Combine per-rank S+ flags: every position was written by exactly one rank, others are 0."""
     if dist.is_initialized() and dist.get_world_size(group) > 1:
-        dist.all_reduce(ext8, op=dist.ReduceOp.MAX, group=group)
+        if _staged(ext8, group):
+            h = ext8.cpu()
+            dist.all_reduce(h, op=dist.ReduceOp.MAX, group=group)
+            ext8.copy_(h)
+        else:
+            dist.all_reduce(ext8, op=dist.ReduceOp.MAX, group=group)
     return ext8
 
 
@@ -75,7 +86,12 @@ def exchange_rows(rows32: torch.Tensor, m: int, d: int, group=None):
     if cw == 0:
         return rows32
     mine = rows32[rank * cw:(rank + 1) * cw].clone()
-    dist.all_gather_into_tensor(rows32[:world * cw], mine, group=group)
+    if _staged(rows32, group):
+        h = torch.empty(world * cw, dtype=rows32.dtype)
+        dist.all_gather_into_tensor(h, mine.cpu(), group=group)
+        rows32[:world * cw].copy_(h)
+    else:
+        dist.all_gather_into_tensor(rows32[:world * cw], mine, group=group)
     return rows32
 
 
