@@ -64,8 +64,11 @@ struct Geo {
 constexpr int kWarps = 16;                // consumer warps = chunks per tile (+1 producer warp)
 // TMA ring depth: 4 stages; at d >= 15 the 2^d-bit task state crowds shared memory (8 KB per task at d = 16),
 // and two stages buy 5 more tasks per CTA (19 -> 24)
+#ifndef SKY_K3_STAGES
+#define SKY_K3_STAGES 4
+#endif
 template <int D>
-constexpr int k3_stages() { return D >= 15 ? 2 : 4; }
+constexpr int k3_stages() { return D >= 15 ? 2 : SKY_K3_STAGES; }
 constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");
