@@ -141,6 +141,9 @@ def parse():
                     help="skycube representation built by each step: the lattice (K4, Fig. 1a, default), the "
                          "HashCube (K5, w=32, Alg. 3 line 13 / Fig. 1b) or both")
     ap.add_argument("--max-level", type=int, default=0, help="partial skycube d' (Appendix A.2); 0 = full")
+    ap.add_argument("--algo", default="mdmc", choices=["mdmc", "sdsc"],
+                    help="mdmc (the product path, default) or the SDSC comparator (Alg. 2, skycube_build_sdsc; "
+                         "1 GPU, host buffers, timed end to end)")
     return ap.parse_args()
 
 
@@ -378,8 +381,39 @@ def measure_e2e(args, x, eng, world, rank, dev, pairs):
             "ms_per_step": t * 1e3, "api": "pipeline.DeviceSkycube (per-rank C-ABI device entry points)"}
 
 
+def run_sdsc(args):
+    """The SDSC comparator (Alg. 2) on the same workload through its C-ABI call (host buffers, H2D and D2H
+    inside the timed region); reported as its own JSON line with "algo": "sdsc"."""
+    import paper_conf_sigmod_boghcsa17_b200 as sky
+    from paper_conf_sigmod_boghcsa17_b200 import build as skybuild
+    skybuild.build()
+    cfg = datagen.config(args.config)
+    x = cfg.data()
+    n, d = x.shape
+    r = sky.skycube_build_sdsc(x, stats=True)  # warm
+    m = r["n_ext"]
+    times, st = [], []
+    for _ in range(max(1, args.steps)):
+        t0 = time.perf_counter()
+        r = sky.skycube_build_sdsc(x, stats=True)
+        times.append(time.perf_counter() - t0)
+        st.append(r["stats"])
+    t = statistics.median(times)
+    pairs = m * (m - 1)
+    print(json.dumps({
+        "algo": "sdsc", "metric": METRIC, "value": pairs / t, "unit": UNIT, "n_gpus": 1, "steps": len(times),
+        "warmup": 1, "ms_per_step": t * 1e3, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "u32", "data": "synthetic",
+        "config": {"workload": workload(cfg), "n": n, "d": d, "n_ext": m, "total_ids": int(r["offsets"][-1])},
+        "phases_ms": {k: statistics.median(s[k] for s in st) for k in ("ms_h2d", "ms_sort", "ms_prefilter", "ms_mdmc", "ms_d2h")},
+        "note": "ms_mdmc is the SDSC lattice traversal (Alg. 2 lines 2-7)"}), flush=True)
+
+
 def main():
     args = parse()
+    if args.algo == "sdsc":
+        run_sdsc(args)
+        return
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -93,6 +93,15 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
 /* Release every buffer of `out` and zero it.  Idempotent; safe on a zeroed struct. */
 void skycube_free(skycube_result *out);
 
+/* SDSC comparator (Alg. 2, §4.2.2): the paper's lattice-based template -- a
+ * top-down traversal where every cuboid delta is computed as a parallel skyline over its cheapest parent's
+ * extended skyline L[parent] U L+[parent] (reading S1: parent = the immediate superset with the fewest
+ * points, ties to the smaller delta').  Same inputs, outputs, conventions and errors as skycube_build_ex
+ * (membership rows, ext_ids and the lattice; opts: device only).  Not the product path: it exists to
+ * compare MDMC with the paper's alternative on the same GPU, and its cost grows with 2^d cuboid passes. */
+skycube_status skycube_build_sdsc(const float *points, int64_t n, int32_t d, const skycube_opts *opts,
+                                  skycube_result *out, skycube_stats *stats);
+
 /* ------------------------------------------------------------------------------------------------
  * HashCube output (Alg. 3 lines 1 and 13, L320; Appendix B.1; Fig. 1b).
  * Point p is represented by B_{p notin S}: 2^d - 1 bits, bit delta-1 set <=> p is dominated in delta

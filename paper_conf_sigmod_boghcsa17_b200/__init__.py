@@ -25,7 +25,7 @@ EXPORTED = (
     "skycube_ctx_create", "skycube_ctx_destroy", "skycube_dev_prepare", "skycube_dev_prefilter",
     "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
     "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_free",
-    "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube",
+    "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc",
 )
 
 
@@ -104,6 +104,8 @@ def lib():
         L.skycube_ctx_launches.restype = I64
         L.skycube_ctx_info.argtypes = [P, ctypes.POINTER(I64), ctypes.POINTER(U32), ctypes.POINTER(U32)]
         L.skycube_ctx_counters.argtypes = [P, P]
+        L.skycube_build_sdsc.argtypes = [P, I64, I32, ctypes.POINTER(Opts), ctypes.POINTER(Result),
+                                          ctypes.POINTER(Stats)]
         L.skycube_build_hashcube.argtypes = [P, I64, I32, U32, ctypes.POINTER(Opts), ctypes.POINTER(HashCube),
                                              ctypes.POINTER(Stats)]
         L.skycube_hashcube_free.argtypes = [ctypes.POINTER(HashCube)]
@@ -115,7 +117,7 @@ def lib():
         for f in ("skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
                   "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_query",
-                  "skycube_ctx_set_max_level", "skycube_dev_hashcube"):
+                  "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -225,6 +227,25 @@ def skycube_build(points: np.ndarray, **kw) -> dict:
         em = r.ext_membership()
         if em is not None:
             out["ext_rows"] = em.copy()
+        if r.stats is not None:
+            out["stats"] = r.stats
+        return out
+
+
+def skycube_build_sdsc(points: np.ndarray, *, device: int = 0, stats: bool = False) -> dict:
+    """The SDSC comparator (Alg. 2) through skycube_build_sdsc: same dict as skycube_build."""
+    pts = np.ascontiguousarray(points, dtype=np.float32)
+    if pts.ndim != 2:
+        raise ValueError("points must be (n, d)")
+    n, d = pts.shape
+    opts = Opts(1, device, 0, 0)
+    res = Result()
+    st = Stats() if stats else None
+    _check(lib().skycube_build_sdsc(pts.ctypes.data_as(ctypes.c_void_p) if n else None, n, d, ctypes.byref(opts),
+                                    ctypes.byref(res), ctypes.byref(st) if st is not None else None))
+    with RawResult(res, st) as r:
+        out = {"rows": r.membership().copy(), "ext_ids": r.ext_ids().copy(), "n_ext": r.n_ext,
+               "offsets": r.offsets().copy(), "ids": r.ids().copy()}
         if r.stats is not None:
             out["stats"] = r.stats
         return out

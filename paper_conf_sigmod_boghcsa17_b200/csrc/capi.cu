@@ -328,6 +328,88 @@ skycube_status skycube_build(const float *points, int64_t n, int32_t d, skycube_
     return skycube_build_ex(points, n, d, nullptr, out, nullptr);
 }
 
+// ------------------------------------------------------------------------------ SDSC comparator (NEXT-3)
+skycube_status skycube_build_sdsc(const float *points, int64_t n, int32_t d, const skycube_opts *opts,
+                                  skycube_result *out, skycube_stats *stats) {
+    if (!out) return fail(SKYCUBE_EINVAL, "out == NULL");
+    std::memset(out, 0, sizeof(*out));
+    if (stats) std::memset(stats, 0, sizeof(*stats));
+    if (d < 1 || d > 16) return fail(SKYCUBE_EINVAL, "d must be in [1, 16]");
+    if (n < 0 || n > INT32_MAX) return fail(SKYCUBE_EINVAL, "n must be in [0, INT32_MAX]");
+    if (n > 0 && !points) return fail(SKYCUBE_EINVAL, "points == NULL");
+    const int device = opts ? opts->device : 0;
+    std::lock_guard<std::mutex> lk(g_mutex);
+    const auto t0 = std::chrono::steady_clock::now();
+    skycube_result r;
+    std::memset(&r, 0, sizeof(r));
+    skycube_status st = guarded([&] {
+        r.d = d;
+        r.n = n;
+        r.words_per_row = sky::words_per_row(d);
+        const uint32_t W = r.words_per_row;
+        const int64_t nsub = (int64_t)1 << d;
+        skycube_ctx *&x = g_ctx[device];
+        if (!x) x = new_ctx(device);
+        else check_device(device);
+        sky::Ctx &c = x->c;
+        const int64_t launches0 = c.L.count;
+        r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
+        if (n == 0) {
+            std::memset(r.cuboid_offsets, 0, sizeof(int64_t) * (nsub + 1));
+            return;
+        }
+        cudaStream_t s = nullptr;
+        Events evs;
+        cudaEvent_t *ev = evs.e;
+        x->input.ensure(sizeof(float) * n * d);
+        SKY_CUDA(cudaEventRecord(ev[0], s));
+        SKY_CUDA(cudaMemcpyAsync(x->input.p, points, sizeof(float) * n * d, cudaMemcpyHostToDevice, s));
+        SKY_CUDA(cudaEventRecord(ev[1], s));
+        sky::prep_run(c, x->input.as<float>(), n, d, s);
+        SKY_CUDA(cudaEventRecord(ev[2], s));
+        x->ext8.ensure(n);
+        sky::prefilter_run(c, 0, 1, x->ext8.as<uint8_t>(), s);
+        sky::ext_build(c, x->ext8.as<uint8_t>(), s);
+        SKY_CUDA(cudaEventRecord(ev[3], s));
+        x->offsets.ensure(sizeof(int64_t) * (nsub + 1));
+        x->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
+        int32_t *d_ids = nullptr;
+        const int64_t total = sky::sdsc_run(c, x->offsets.as<int64_t>(), x->membership.as<uint32_t>(), s, &d_ids);
+        SKY_CUDA(cudaEventRecord(ev[4], s));
+        const int64_t m = c.m;
+        r.n_ext = m;
+        r.ext_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (m > 0 ? m : 1));
+        r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
+        r.cuboid_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (total > 0 ? total : 1));
+        if (m) SKY_CUDA(cudaMemcpyAsync(r.ext_ids, c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaMemcpyAsync(r.membership, x->membership.p, sizeof(uint32_t) * (size_t)n * W, cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaMemcpyAsync(r.cuboid_offsets, x->offsets.p, sizeof(int64_t) * (nsub + 1), cudaMemcpyDeviceToHost, s));
+        if (total) SKY_CUDA(cudaMemcpyAsync(r.cuboid_ids, d_ids, sizeof(int32_t) * total, cudaMemcpyDeviceToHost, s));
+        SKY_CUDA(cudaEventRecord(ev[5], s));
+        SKY_CUDA(cudaStreamSynchronize(s));
+        SKY_CUDA(cudaGetLastError());
+        if (stats) {
+            stats->ms_h2d = ev_ms(ev[0], ev[1]);
+            stats->ms_sort = ev_ms(ev[1], ev[2]);
+            stats->ms_prefilter = ev_ms(ev[2], ev[3]);
+            stats->ms_mdmc = ev_ms(ev[3], ev[4]);  // the SDSC lattice traversal
+            stats->ms_d2h = ev_ms(ev[4], ev[5]);
+            stats->n_ext = m;
+            stats->pairs = m * (m > 0 ? m - 1 : 0);
+            stats->total_ids = total;
+            stats->kernel_launches = (int32_t)(c.L.count - launches0);
+        }
+    });
+    if (st != SKYCUBE_OK) {
+        skycube_free(&r);
+        return st;
+    }
+    if (stats)
+        stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = r;
+    return SKYCUBE_OK;
+}
+
 // ------------------------------------------------------------------------------ HashCube (NEXT-1/4)
 void skycube_hashcube_free(skycube_hashcube *hc) {
     if (!hc) return;
@@ -455,6 +537,7 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
                            &ctx->membership, &ctx->offsets, &ctx->ids})
         b->release();
     c.hc.release();
+    c.release_sdsc();
     if (ctx->side) cudaStreamDestroy(ctx->side);
     if (ctx->ev_ext) cudaEventDestroy(ctx->ev_ext);
     if (ctx->ev_side) cudaEventDestroy(ctx->ev_side);

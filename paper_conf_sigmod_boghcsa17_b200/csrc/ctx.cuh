@@ -93,6 +93,15 @@ struct Ctx {
     DevBuf counters;    // u64 [8]: K1 box tests, K1 pair tests, K3 box tests, K3 pair tests, K3 misses
     DevBuf scan64_tmp;
     HashCubeState hc;
+    // SDSC comparator (sdsc.cu)
+    DevBuf sdsc_prev, sdsc_next, sdsc_ids_tmp, sdsc_tab, sdsc_items, sdsc_keys, sdsc_vals, sdsc_keys_alt, sdsc_vals_alt,
+        sdsc_counts, sdsc_scan, sdsc_status, sdsc_flags, sdsc_cnt, sdsc_lat, sdsc_ids;
+    void release_sdsc() {
+        for (DevBuf *b : {&sdsc_prev, &sdsc_next, &sdsc_ids_tmp, &sdsc_tab, &sdsc_items, &sdsc_keys, &sdsc_vals,
+                          &sdsc_keys_alt, &sdsc_vals_alt, &sdsc_counts, &sdsc_scan, &sdsc_status, &sdsc_flags,
+                          &sdsc_cnt, &sdsc_lat, &sdsc_ids})
+            b->release();
+    }
 };
 
 // prep.cu
@@ -110,6 +119,9 @@ void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cu
 void membership_zero_outside(Ctx &c, uint32_t *membership, cudaStream_t st);
 void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
                      cudaStream_t st);
+// sdsc.cu: Alg. 2 over the installed S+; lattice into d_offsets / *d_ids (context-owned), rows into
+// d_membership (nullable); returns the number of ids
+int64_t sdsc_run(Ctx &c, int64_t *d_offsets, uint32_t *d_membership, cudaStream_t st, int32_t **d_ids);
 // k5_hashcube.cu
 int64_t hashcube_words(int d, uint32_t w);
 void hashcube_build(Ctx &c, const uint32_t *rows32, uint32_t w, cudaStream_t st);
