@@ -12,9 +12,10 @@
 // for every q of the chunk, so bit Mbox set in the probe set proves the whole chunk adds nothing (Λ4 on a
 // leaf range: the paper's filter on path labels, L320-328, with the tree's global pivots).
 //
-// A CTA holds up to NT tasks (codes + state in shared memory) and streams every chunk once (TMA ring fed by
-// one producer warp); each of the 16 consumer warps takes one chunk per tile, one competitor per lane in
-// registers:
+// Design A (k3_mdmc_kernel): a CTA holds up to NT tasks (codes + state in shared memory) and streams every
+// chunk once (TMA ring fed by one producer warp); each of the 16 consumer warps takes one chunk per tile, one
+// competitor per lane in registers.  Design O (k3_owner_kernel, further below) swaps the roles: a warp owns
+// 32 tasks and takes a share of every tile's chunks.  Both run the same three passes:
 //   box pass   lane l tests task 32g+l against the chunk corner (SWAR over 16-bit code lanes with guard
 //              bits, gathered to a d-bit mask with a byte permute and a carry-free multiply per 4
 //              dimensions) and probes the task's state; a ballot gives the tasks whose chunk must be opened;
@@ -476,6 +477,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         };
         auto box_test = [&](int tt, uint32_t &Mb) {
             uint32_t le[G::CW];
+            // scalar loads from the odd-stride row copy: conflict-free across the 32 task lanes (two LDS.128
+            // from the 16-byte-stride copy measured 5% slower at H: 4+ wavefronts each, longer latency)
 #pragma unroll
             for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
             Mb = gather_mask<G::NG>(le);
