@@ -61,8 +61,11 @@ typedef struct {
 } skycube_result;
 
 typedef struct {
-    int32_t num_gpus;     /* reserved for the single-process multi-GPU path; 0 or 1 = one GPU */
-    int32_t device;       /* CUDA device ordinal to use */
+    int32_t num_gpus;     /* 0 or 1 = one GPU; k > 1 = single-process sharding over devices device .. device+k-1:
+                             prepare replicated, K1 blocks and K3 task groups split k ways, S+ flags and rows
+                             gathered on `device` by peer copies (NVLink); same output bytes as one GPU.
+                             ENODEV if fewer devices are visible; not with SKYCUBE_EXT_MEMBERSHIP (EINVAL) */
+    int32_t device;       /* CUDA device ordinal to use (the first one when num_gpus > 1) */
     uint32_t flags;       /* SKYCUBE_* flags */
     int32_t max_level;    /* partial skycube (Appendix A.2): 0 = full skycube; d' in [1, d] =
                              only the subspaces with |delta| <= d' are computed and reported -- membership

@@ -200,14 +200,14 @@ class RawResult:
 
 
 def skycube_build_raw(points: np.ndarray, *, device: int = 0, lists: bool = True, ext_membership: bool = False,
-                      stats: bool = False, max_level: int = 0) -> RawResult:
+                      stats: bool = False, max_level: int = 0, num_gpus: int = 1) -> RawResult:
     """Call skycube_build_ex on a host (n, d) float32 array; returns the owning RawResult.
     max_level = d' > 0 computes the partial skycube (|delta| <= d' only, Appendix A.2)."""
     pts = np.ascontiguousarray(points, dtype=np.float32)
     if pts.ndim != 2:
         raise ValueError("points must be (n, d)")
     n, d = pts.shape
-    opts = Opts(1, device, (0 if lists else NO_LISTS) | (EXT_MEMBERSHIP if ext_membership else 0), max_level)
+    opts = Opts(num_gpus, device, (0 if lists else NO_LISTS) | (EXT_MEMBERSHIP if ext_membership else 0), max_level)
     res = Result()
     st = Stats() if stats else None
     _check(lib().skycube_build_ex(pts.ctypes.data_as(ctypes.c_void_p) if n else None, n, d, ctypes.byref(opts),

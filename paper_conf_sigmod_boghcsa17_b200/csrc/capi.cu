@@ -8,13 +8,14 @@
 #include <map>
 #include <mutex>
 #include <unordered_map>
+#include <vector>
 
 #include "../../include/skycube.h"
 #include "ctx.cuh"
 
 struct skycube_ctx {
     sky::Ctx c;
-    sky::DevBuf input, ext8, rows32, ext_rows32, membership, offsets, ids;
+    sky::DevBuf input, ext8, rows32, ext_rows32, membership, offsets, ids, flag_stage;
     cudaStream_t side = nullptr;  // non-blocking stream for work that overlaps the main (default) stream
     cudaEvent_t ev_ext = nullptr, ev_side = nullptr;
 };
@@ -89,6 +90,7 @@ struct PinnedPool {
 PinnedPool g_pool;
 
 std::map<int, skycube_ctx *> g_ctx;  // one cached context per device for skycube_build*
+std::map<int, skycube_ctx *> g_mctx; // multi-GPU builds: one context per (rank, device)
 
 void check_device(int device) {
     int count = 0;
@@ -186,6 +188,163 @@ struct Events {
     }
 };
 
+
+// Single-process multi-GPU build: num_gpus = k logical ranks on devices first .. first+k-1
+// (SKYCUBE_SHARE_DEVICES=1 lets ranks share devices round-robin -- the multi-rank logic on one GPU, tests).
+//   every rank: H2D of the points, K0/K2 prepare (replicated, deterministic)
+//   rank g:     K1 on the prefilter blocks b = g (mod k); the k flag vectors are gathered on rank 0 by
+//               peer copies (NVLink), OR-combined and broadcast back; every rank installs S+
+//   rank g:     K3 on its contiguous range of 32-task groups; the row ranges are gathered on rank 0
+//   rank 0:     K4 (membership, lattice) and the D2H.
+// The output bytes are those of the single-GPU build (every kernel's result is scheduling-independent).
+skycube_status build_multi(const float *points, int64_t n, int d, int first, int k, int max_level, bool lists,
+                           skycube_result *out, skycube_stats *stats) {
+    std::lock_guard<std::mutex> lk(g_mutex);
+    const auto t0 = std::chrono::steady_clock::now();
+    skycube_result r;
+    std::memset(&r, 0, sizeof(r));
+    skycube_status st = guarded([&] {
+        int count = 0;
+        if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) {
+            cudaGetLastError();
+            throw sky::Error{SKYCUBE_ENODEV, "no CUDA device visible"};
+        }
+        const char *share_env = getenv("SKYCUBE_SHARE_DEVICES");
+        const bool share = share_env && share_env[0] == '1';
+        if (!share && first + k > count)
+            throw sky::Error{SKYCUBE_ENODEV, "num_gpus exceeds the visible devices after `device`"};
+        std::vector<int> dev(k);
+        std::vector<skycube_ctx *> xs(k);
+        for (int g = 0; g < k; g++) {
+            dev[g] = (first + g) % count;
+            check_device(dev[g]);
+            skycube_ctx *&x = g_mctx[(g << 8) | dev[g]];
+            if (!x) x = new_ctx(dev[g]);
+            xs[g] = x;
+        }
+        for (int g = 1; g < k; g++) {  // NVLink peer access between rank 0 and every other device
+            if (dev[g] == dev[0]) continue;
+            int can = 0;
+            cudaDeviceCanAccessPeer(&can, dev[0], dev[g]);
+            if (can) {
+                SKY_CUDA(cudaSetDevice(dev[0]));
+                if (cudaDeviceEnablePeerAccess(dev[g], 0) != cudaSuccess) cudaGetLastError();
+            }
+        }
+        r.d = d;
+        r.n = n;
+        r.words_per_row = sky::words_per_row(d);
+        const uint32_t W = r.words_per_row;
+        const int64_t nsub = (int64_t)1 << d;
+        auto sync_all = [&] {
+            for (int g = 0; g < k; g++) {
+                SKY_CUDA(cudaSetDevice(dev[g]));
+                SKY_CUDA(cudaDeviceSynchronize());
+            }
+        };
+        int64_t launches0 = 0;
+        for (int g = 0; g < k; g++) launches0 += xs[g]->c.L.count;
+        const auto tp0 = std::chrono::steady_clock::now();
+        // prepare (replicated) + the rank's prefilter blocks
+        for (int g = 0; g < k; g++) {
+            skycube_ctx *x = xs[g];
+            SKY_CUDA(cudaSetDevice(dev[g]));
+            x->input.ensure(sizeof(float) * n * d);
+            SKY_CUDA(cudaMemcpyAsync(x->input.p, points, sizeof(float) * n * d, cudaMemcpyHostToDevice, nullptr));
+            sky::prep_run(x->c, x->input.as<float>(), n, d, nullptr);
+            x->ext8.ensure(n);
+            SKY_CUDA(cudaMemsetAsync(x->ext8.p, 0, n, nullptr));
+            sky::prefilter_run(x->c, g, k, x->ext8.as<uint8_t>(), nullptr);
+        }
+        sync_all();
+        // gather the flags on rank 0, OR, broadcast
+        skycube_ctx *x0 = xs[0];
+        SKY_CUDA(cudaSetDevice(dev[0]));
+        x0->flag_stage.ensure((size_t)n * k);
+        for (int g = 0; g < k; g++)
+            SKY_CUDA(cudaMemcpyPeerAsync(x0->flag_stage.as<uint8_t>() + (size_t)g * n, dev[0], xs[g]->ext8.p, dev[g], n, nullptr));
+        sky::or_flags(x0->c, x0->flag_stage.as<uint8_t>(), k, n, x0->ext8.as<uint8_t>(), nullptr);
+        for (int g = 1; g < k; g++)
+            SKY_CUDA(cudaMemcpyPeerAsync(xs[g]->ext8.p, dev[g], x0->ext8.p, dev[0], n, nullptr));
+        sync_all();
+        const auto tp1 = std::chrono::steady_clock::now();
+        for (int g = 0; g < k; g++) {
+            SKY_CUDA(cudaSetDevice(dev[g]));
+            sky::ext_build(xs[g]->c, xs[g]->ext8.as<uint8_t>(), nullptr);
+        }
+        const int64_t m = x0->c.m;
+        const int64_t groups = sky::ceil_div(m, 32), gpr = sky::ceil_div(groups, k);
+        const size_t grp_words = (size_t)W * 32;
+        const size_t rows_words = (size_t)std::max<int64_t>(groups, 1) * grp_words;
+        for (int g = 0; g < k; g++) {
+            skycube_ctx *x = xs[g];
+            SKY_CUDA(cudaSetDevice(dev[g]));
+            x->rows32.ensure(sizeof(uint32_t) * rows_words);
+            const int64_t j0 = std::min<int64_t>(m, g * gpr * 32), j1 = std::min<int64_t>(m, (g + 1) * gpr * 32);
+            x->c.max_level = max_level;
+            if (j1 > j0) sky::mdmc_run(x->c, j0, j1, x->rows32.as<uint32_t>(), nullptr, nullptr);
+        }
+        sync_all();
+        const auto tp2 = std::chrono::steady_clock::now();
+        SKY_CUDA(cudaSetDevice(dev[0]));
+        for (int g = 1; g < k; g++) {
+            const int64_t j0 = std::min<int64_t>(m, g * gpr * 32), j1 = std::min<int64_t>(m, (g + 1) * gpr * 32);
+            if (j1 <= j0) continue;
+            const size_t w0 = (size_t)(j0 / 32) * grp_words, w1 = (size_t)sky::ceil_div(j1, 32) * grp_words;
+            SKY_CUDA(cudaMemcpyPeerAsync(x0->rows32.as<uint32_t>() + w0, dev[0], xs[g]->rows32.as<uint32_t>() + w0, dev[g],
+                                         sizeof(uint32_t) * (w1 - w0), nullptr));
+        }
+        sky::Ctx &c = x0->c;
+        x0->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
+        sky::compact_membership(c, x0->rows32.as<uint32_t>(), x0->membership.as<uint32_t>(), nullptr);
+        int64_t total = 0;
+        if (lists) {
+            x0->offsets.ensure(sizeof(int64_t) * (nsub + 1));
+            sky::compact_lattice(c, x0->rows32.as<uint32_t>(), x0->offsets.as<int64_t>(), nullptr, &total, nullptr);
+            x0->ids.ensure(sizeof(int32_t) * (total > 0 ? total : 1));
+            sky::compact_lattice(c, x0->rows32.as<uint32_t>(), x0->offsets.as<int64_t>(), x0->ids.as<int32_t>(), &total,
+                                 nullptr);
+        }
+        r.n_ext = m;
+        r.ext_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (m > 0 ? m : 1));
+        r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
+        if (m) SKY_CUDA(cudaMemcpyAsync(r.ext_ids, c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, nullptr));
+        SKY_CUDA(cudaMemcpyAsync(r.membership, x0->membership.p, sizeof(uint32_t) * (size_t)n * W, cudaMemcpyDeviceToHost,
+                                 nullptr));
+        if (lists) {
+            r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
+            r.cuboid_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (total > 0 ? total : 1));
+            SKY_CUDA(cudaMemcpyAsync(r.cuboid_offsets, x0->offsets.p, sizeof(int64_t) * (nsub + 1), cudaMemcpyDeviceToHost,
+                                     nullptr));
+            if (total)
+                SKY_CUDA(cudaMemcpyAsync(r.cuboid_ids, x0->ids.p, sizeof(int32_t) * total, cudaMemcpyDeviceToHost, nullptr));
+        }
+        SKY_CUDA(cudaDeviceSynchronize());
+        SKY_CUDA(cudaGetLastError());
+        const auto tp3 = std::chrono::steady_clock::now();
+        if (stats) {  // host clock per phase (several devices)
+            auto ms = [](auto a, auto b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
+            stats->ms_sort = ms(tp0, tp1);  // H2D + prepare + prefilter + flag exchange
+            stats->ms_mdmc = ms(tp1, tp2);  // S+ install + K3
+            stats->ms_compact = ms(tp2, tp3);  // row gather + K4 + D2H
+            stats->n_ext = m;
+            stats->pairs = m * (m > 0 ? m - 1 : 0);
+            stats->total_ids = total;
+            int64_t launches = 0;
+            for (int g = 0; g < k; g++) launches += xs[g]->c.L.count;
+            stats->kernel_launches = (int32_t)(launches - launches0);
+        }
+    });
+    if (st != SKYCUBE_OK) {
+        skycube_free(&r);
+        return st;
+    }
+    if (stats)
+        stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = r;
+    return SKYCUBE_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -227,6 +386,12 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
     const int device = opts ? opts->device : 0;
     const int max_level = opts ? opts->max_level : 0;
     if (max_level < 0 || max_level > d) return fail(SKYCUBE_EINVAL, "max_level must be in [0, d]");
+    const int num_gpus = opts ? opts->num_gpus : 1;
+    if (num_gpus < 0 || num_gpus > 64) return fail(SKYCUBE_EINVAL, "num_gpus must be in [0, 64]");
+    if (num_gpus > 1 && n > 0) {
+        if (flags & SKYCUBE_EXT_MEMBERSHIP) return fail(SKYCUBE_EINVAL, "EXT_MEMBERSHIP is single-GPU only");
+        return build_multi(points, n, d, device, num_gpus, max_level, !(flags & SKYCUBE_NO_LISTS), out, stats);
+    }
     std::lock_guard<std::mutex> lk(g_mutex);
     const auto t0 = std::chrono::steady_clock::now();
     skycube_result r;

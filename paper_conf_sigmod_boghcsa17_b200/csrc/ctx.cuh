@@ -107,6 +107,7 @@ struct Ctx {
 // prep.cu
 void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st);
 void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st);
+void or_flags(Ctx &c, const uint8_t *stage, int k, int64_t n, uint8_t *out, cudaStream_t st);
 // k1_prefilter.cu
 void prefilter_run(Ctx &c, int64_t tile_offset, int64_t tile_step, uint8_t *d_ext_sorted, cudaStream_t st);
 // k3_mdmc.cu

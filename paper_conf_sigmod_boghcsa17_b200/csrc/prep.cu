@@ -245,6 +245,21 @@ void pad_ord(uint32_t *ord, int64_t from, int64_t to, int d, cudaStream_t st, La
 
 }  // namespace
 
+// out[s] = OR over the k per-device flag vectors stage[g * n + s] (single-process multi-GPU prefilter)
+__global__ void or_flags_kernel(const uint8_t *__restrict__ stage, int k, int64_t n, uint8_t *__restrict__ out) {
+    const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= n) return;
+    uint8_t v = 0;
+    for (int g = 0; g < k; g++) v |= stage[(int64_t)g * n + s];
+    out[s] = v;
+}
+
+void or_flags(Ctx &c, const uint8_t *stage, int k, int64_t n, uint8_t *out, cudaStream_t st) {
+    or_flags_kernel<<<blocks_for(n, 256), 256, 0, st>>>(stage, k, n, out);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
 void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) {
     c.n = n;
     c.d = d;

@@ -117,3 +117,14 @@ def test_hashcube_query_host_logic_fig1b(lib):
                                               ctypes.byref(cnt)) == sky.OK
             assert out[:cnt.value].tolist() == gold["lattice"][str(delta)], (w, delta)
         assert lib.skycube_hashcube_query(ctypes.byref(hc), 8, None, ctypes.byref(cnt)) == sky.EINVAL
+
+
+def test_num_gpus_validation_without_gpu(lib):
+    pts = np.zeros((4, 3), np.float32)
+    p = pts.ctypes.data_as(ctypes.c_void_p)
+    res = sky.Result()
+    assert lib.skycube_build_ex(p, 4, 3, ctypes.byref(sky.Opts(-1, 0, 0, 0)), ctypes.byref(res), None) == sky.EINVAL
+    assert lib.skycube_build_ex(p, 4, 3, ctypes.byref(sky.Opts(2, 0, sky.EXT_MEMBERSHIP, 0)), ctypes.byref(res),
+                                None) == sky.EINVAL
+    # no device in this container: the multi-GPU path reports ENODEV, never a CPU fallback
+    assert lib.skycube_build_ex(p, 4, 3, ctypes.byref(sky.Opts(2, 0, 0, 0)), ctypes.byref(res), None) == sky.ENODEV

@@ -79,3 +79,29 @@ def test_multirank_bytes_equal_single_rank(world, name):
         for k in ("word_offsets", "keys", "key_offsets", "ids"):
             got = r["hc_" + k].view(np.uint32) if k == "keys" else r["hc_" + k]
             assert np.array_equal(got, want_hc[k]), (rank, k)
+
+
+@pytest.mark.parametrize("k,name", [(2, "C3I"), (3, "A-small"), (4, "ct-small"), (2, "C2")])
+def test_capi_num_gpus_bytes_equal_single_gpu(monkeypatch, k, name):
+    """The C-ABI's single-process multi-GPU path (skycube_opts.num_gpus = k): k logical ranks, here sharing
+    the one GPU (SKYCUBE_SHARE_DEVICES=1), with the flag OR-combine, the peer-copy gathers and the sharded
+    K1/K3 ranges; every output byte must equal the one-GPU build."""
+    import torch
+    import paper_conf_sigmod_boghcsa17_b200 as sky
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    if name == "A-small":
+        x = datagen.generate("A", 60000, 10, 91)
+    elif name == "ct-small":
+        x = datagen.generate("ct", 80000, 10, 92)
+    else:
+        x = datagen.config(name).data()
+    want = sky.skycube_build(x)
+    monkeypatch.setenv("SKYCUBE_SHARE_DEVICES", "1")
+    with sky.skycube_build_raw(x, num_gpus=k, stats=True) as r:
+        assert np.array_equal(r.membership(), want["rows"])
+        assert np.array_equal(r.ext_ids(), want["ext_ids"])
+        assert np.array_equal(r.offsets(), want["offsets"]) and np.array_equal(r.ids(), want["ids"])
+        assert r.stats["kernel_launches"] > 0
+    with sky.skycube_build_raw(x, num_gpus=k, max_level=3) as r:
+        assert np.array_equal(r.membership(), sky.skycube_build(x, max_level=3)["rows"])
