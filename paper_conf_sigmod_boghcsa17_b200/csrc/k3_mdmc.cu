@@ -786,7 +786,20 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
-    const int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
+    int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
+    if (tpc == C::NT) {
+        // Wave quantisation (one CTA per SM): a CTA's time grows with its task groups (the box pass walks
+        // every group of every chunk) plus about one group's worth of per-tile work, so pick the task count
+        // that minimises waves x (groups + 1) — e.g. C3I: 4 waves of 9 groups -> 4 waves of 8.
+        auto cost = [&](int64_t t) { return ceil_div(ceil_div(range, t), (int64_t)c.num_sms) * (ceil_div(t, (int64_t)32) + 1); };
+        int64_t best = cost(tpc);
+        for (int t = (C::NT / 32) * 32; t >= 32; t -= 32)
+            if (cost(t) < best) {
+                best = cost(t);
+                tpc = t;
+            }
+    }
+    if (const char *e = getenv("SKYCUBE_K3_TPC"); e && *e) tpc = std::max(1, std::min<int>(C::NT, atoi(e)));
     const size_t smem = C::smem_bytes(tpc);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
