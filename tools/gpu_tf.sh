@@ -1,5 +1,6 @@
 #!/bin/bash
-# GPU-box helper: K3 tile-filter / chunk-key A/B.  GPU tests first (TESTS=0 skips), then bench lines for
+# GPU-box helper: K3 tile-filter / chunk-key A/B (the experiment recorded in DESIGN.md §5; the code it
+# drove was reverted, so at HEAD SKYCUBE_K3_TILEFILTER / SKYCUBE_K3_KEYSHIFT have no effect).  GPU tests first (TESTS=0 skips), then bench lines for
 # CONFIGS under each (SKYCUBE_K3_TILEFILTER, SKYCUBE_K3_KEYSHIFT) pair in VARIANTS ("tf:shift ...").
 mkdir -p gpurun_out
 if [ "${TESTS:-1}" != 0 ]; then
