@@ -5,6 +5,8 @@ n=1M d=12 anticorr, 1/2/4/8 B200").
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config H] [--impl ours|reference]
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
 
+`--gpus N` without torchrun re-launches itself as N ranks under torch.distributed.run (one process per GPU).
+
 One step = one whole skycube build (K0 validate -> key sort -> K2 codes -> K1 prefilter -> S+ ->
 K3 MDMC -> K4 compaction into membership rows and the per-subspace id lists) over the synthetic
 workload, input resident in HBM.  value = dominance tests/s = n_ext*(n_ext-1) / (step time, max over
@@ -41,12 +43,55 @@ def algorithmic_ops_per_test(d: int) -> int:
     return d + 2
 
 
-def alu_peak_ops(sm_mhz: float, sms: int = 148) -> float:
-    """Integer issue peak (DESIGN.md §Roofline): each SMSP issues at most one warp instruction per clock;
-    integer work runs on the ALU pipe (IADD3/LOP3/SHF/PRMT, 16 lanes/SMSP) and on the FMA pipe
-    (IMAD/IMAD.IADD, 16 lanes/SMSP) (B300_MICROARCH.md "Pipe rates"), so 4 x 32 = 128 integer lane-ops
-    per SM per clock."""
-    return sms * 128 * sm_mhz * 1e6
+INTPEAK = os.path.join(ROOT, "profiles", "r02_intpeak.json")
+
+
+def int_peaks(sm_mhz: float, sms: int = 148):
+    """Integer lane-op peaks at the SM clock of the run, from the MEASURED microbenchmark
+    (tools/intpeak.cu on one B200, profiles/r02_intpeak.json): lane-ops per SM per clock of (a) the ALU pipe
+    alone (LOP3/IADD3/PRMT/SHF chains) and (b) ALU + FMA pipes together (LOP3 interleaved with IMAD, the
+    one-warp-instruction-per-SMSP-per-clock issue bound).  Falls back to the B300_MICROARCH pipe rates
+    (rt_SMSP = 2 per pipe: 64 and 128 lanes/SM/clk) only if the measurement file is absent, and says so."""
+    try:
+        with open(INTPEAK) as f:
+            m = json.load(f)
+        alu, mix = m["alu"]["lane_ops_per_sm_per_clk"], m["mix"]["lane_ops_per_sm_per_clk"]
+        basis = (f"measured (profiles/r02_intpeak.json: {alu:.1f} ALU-only and {mix:.1f} ALU+FMA integer lane-ops "
+                 f"per SM per clock) x {sms} SMs x {sm_mhz:.0f} MHz (median SM clock of this run)")
+    except Exception:
+        alu, mix = 64.0, 128.0
+        basis = f"FALLBACK (no profiles/r02_intpeak.json): B300_MICROARCH pipe rates 64 / 128 lanes/SM/clk x {sms} x {sm_mhz:.0f} MHz"
+    return alu * sms * sm_mhz * 1e6, mix * sms * sm_mhz * 1e6, basis
+
+
+def golden_fullsize(config: str):
+    """The offline full-size Oracle B record of a config (tests/golden/fullsize_digests.json, written by
+    tools/oracle_digest.py, which calls only oracle/), or None."""
+    try:
+        with open(os.path.join(ROOT, "tests", "golden", "fullsize_digests.json")) as f:
+            return json.load(f)["configs"].get(config)
+    except Exception:
+        return None
+
+
+def cpu_model() -> str:
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def config_dict(cfg, args, world: int, m: int, total_ids) -> dict:
+    """The `config` object of both arms (identical keys, so the driver can match them)."""
+    return {"workload": workload(cfg), "n": cfg.n, "d": cfg.d, "n_ext": m, "pairs": m * (m - 1),
+            "total_ids": total_ids, "output": args.output, "max_level": args.max_level or cfg.d,
+            "l2": "256 MB buffer written between timed steps",
+            "parallelism": (f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, "
+                            f"rows all-gathered" if world > 1 else "dp1")}
 
 
 def ncu_traffic(config: str, kernel: str):
@@ -59,6 +104,19 @@ def ncu_traffic(config: str, kernel: str):
         return int(e["dram_read_bytes"]) + int(e["dram_write_bytes"]), e.get("source")
     except Exception:
         return None, None
+
+
+def ncu_instructions(config: str, kernel: str):
+    """smsp__inst_executed.sum (warp instructions) of one launch of `kernel` at `config` and the tests the
+    same launch executed (device counters), from the committed ncu capture summarised in profiles/traffic.json."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            e = json.load(f)[config][kernel]
+        if "warp_instructions" in e and "tests" in e:
+            return e
+    except Exception:
+        pass
+    return None
 
 
 def workload(cfg) -> str:
@@ -132,7 +190,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="H", choices=sorted(datagen.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
@@ -184,19 +242,30 @@ def run_reference(args):
         if i >= args.warmup:
             times.append((full_s, k, t, est_next, thr))
     full = statistics.median([a[0] for a in times])
-    est_next = times[0][3]
-    value = est_next * (est_next - 1) / full
+    gold = golden_fullsize(args.config)
+    if gold is not None and not args.max_level:
+        # exact |S+| and id count of this workload, computed offline by the oracle itself (tools/oracle_digest.py)
+        m, total_ids, m_src = gold["n_ext"], gold["total_ids"], "exact (tests/golden/fullsize_digests.json, Oracle B)"
+    else:
+        m, total_ids, m_src = times[0][3], None, "estimated from the sample's S+ bits"
+    value = m * (m - 1) / full
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": full * 1e3, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": workload(cfg), "n": cfg.n, "d": cfg.d, "n_ext_estimated": est_next},
+        "config": config_dict(cfg, args, args.gpus, m, total_ids),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": times[0][4], "kind": "oracle",
-                         "sample": f"Oracle B (oracle/skycube_oracle.c) rows for {times[0][1]} uniformly sampled "
-                                   f"points of {cfg.n} per step ({times[0][2]:.1f} s), extrapolated x n/sample; "
-                                   f"n_ext estimated from the sample's S+ bits"},
+                         "cpu_model": cpu_model(),
+                         "sample": f"Oracle B (oracle/skycube_oracle.c, -O2) rows for {times[0][1]} uniformly sampled "
+                                   f"points of {cfg.n} per step ({times[0][2]:.1f} s on {times[0][4]} threads), "
+                                   f"extrapolated x n/sample; n_ext {m_src}"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
+    if gold is not None:
+        o = gold["oracle"]
+        line["cpu_baseline"]["full_run"] = (f"the whole workload was run once by tools/oracle_digest.py: Oracle B over all "
+                                            f"{cfg.n} points in {o['rows_b_wall_s']:.0f} s on {o['threads']} threads "
+                                            f"({o['cpu_model']}, -O3 -march=native build of the same source)")
     print(json.dumps(line), flush=True)
 
 
@@ -280,6 +349,9 @@ def run_ours(args):
     if not args.no_e2e:
         e2e = measure_e2e(args, x, eng, world, rank, dev, pairs)
 
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
     if rank != 0:
         return
     clocks = clk.summary()
@@ -290,34 +362,43 @@ def run_ours(args):
     tests = work["k3_box"] + work.get("k3_sub", 0) + work["k3_pair"]
     ops = tests * algorithmic_ops_per_test(d)
     achieved = ops / (mdmc_ms / 1e3) / 1e12
-    peak = alu_peak_ops(sm_mhz) / 1e12
+    peak_alu, peak_mix, peak_basis = int_peaks(sm_mhz)
+    peak = peak_mix / 1e12
     traffic, traffic_src = ncu_traffic(args.config, "k3_mdmc") if world == 1 else (None, None)
+    conf = config_dict(cfg, args, world, m, total_ids)
+    if hc_w:
+        conf["output"] += f" (w=32, {hc_ids} stored ids)"
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": workload(cfg), "n": n, "d": d, "n_ext": m, "pairs": pairs, "total_ids": total_ids,
-                   "output": args.output + (f" (w=32, {hc_ids} stored ids)" if hc_w else ""),
-                   "max_level": args.max_level or d,
-                   "l2": "256 MB buffer written between timed steps",
-                   "parallelism": f"dp{world}: K1 tiles and K3 task groups sharded, S+ flags all-reduced, rows all-gathered"},
+        "config": conf,
         "phases_ms": phase,
         "work_per_step": work,
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tlane-op/s",
-                     "frac": achieved / peak, "traffic": traffic, "traffic_unit": "bytes (DRAM read+write per launch)",
+                     "frac": achieved / peak, "frac_alu_only": achieved / (peak_alu / 1e12),
+                     "traffic": traffic, "traffic_unit": "bytes (DRAM read+write per launch)",
                      "traffic_source": traffic_src,
                      "kernel": "k3_mdmc", "ops_per_test": algorithmic_ops_per_test(d), "tests": tests,
-                     "peak_basis": f"148 SM x 128 integer lanes/clk (ALU+FMA pipes, 1 warp-inst/SMSP/clk) x {sm_mhz:.0f} MHz "
-                                   f"(median SM clock under load)"},
+                     "resolved_pairs": pairs,
+                     "peak_basis": "peak = ALU+FMA integer issue bound; frac_alu_only against the ALU pipe alone; "
+                                   + peak_basis},
         "clocks": clocks,
     }
+    ins = ncu_instructions(args.config, "k3_mdmc") if world == 1 else None
+    if ins:
+        line["roofline"]["ncu_lane_instructions_per_test"] = 32.0 * ins["warp_instructions"] / ins["tests"]
+        line["roofline"]["ncu_lane_instructions_per_resolved_pair"] = 32.0 * ins["warp_instructions"] / pairs
+        line["roofline"]["ncu_alu_pipe_pct"] = ins.get("alu_pipe_pct")
+        line["roofline"]["ncu_source"] = ins.get("source")
     if e2e is not None:
         line["e2e"] = e2e
     if not args.no_cpu and world == 1 or (not args.no_cpu and rank == 0 and world == 1):
         full_s, k, t, est_next, thr = oracle_sample_time(x, args.cpu_seconds)
         cpu_value = pairs / full_s
         line["cpu_baseline"] = {"value": cpu_value, "unit": UNIT, "cores": thr, "kind": "oracle",
+                                "cpu_model": cpu_model(),
                                 "sample": f"Oracle B rows for {k} uniformly sampled points of {n} "
                                           f"({t:.1f} s on {thr} threads), extrapolated x n/sample to "
                                           f"{full_s:.0f} s for the whole build"}
@@ -412,8 +493,37 @@ def run_sdsc(args):
         "note": "ms_mdmc is the SDSC lattice traversal (Alg. 2 lines 2-7)"}), flush=True)
 
 
+def spawn_ranks(args) -> int:
+    """`bench.py --gpus N` without a torchrun environment: re-launch this script as N ranks (one process per
+    GPU) under torch.distributed.run on 127.0.0.1, with NCCL_DEBUG=INFO so the communicator lines show the N
+    ranks.  The ranks' JSON line (rank 0) goes to stdout; every other line of theirs to stderr."""
+    import socket
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} requested but only {have} CUDA device(s) are visible\n")
+        return 2
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("OMP_NUM_THREADS", "4")
+    proc = subprocess.Popen(cmd, env=env, stdout=subprocess.PIPE, text=True, bufsize=1)
+    for line in proc.stdout:
+        (sys.stdout if line.lstrip().startswith("{") else sys.stderr).write(line)
+        sys.stdout.flush()
+    return proc.wait()
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "LOCAL_RANK" not in os.environ and args.impl == "ours" and args.algo == "mdmc":
+        sys.exit(spawn_ranks(args))
+    if "WORLD_SIZE" in os.environ and args.gpus > 1 and int(os.environ["WORLD_SIZE"]) != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={os.environ['WORLD_SIZE']}")
     if args.algo == "sdsc":
         run_sdsc(args)
         return

@@ -3,21 +3,21 @@
  * "Template Skycube Algorithms for Heterogeneous Parallelism on Multicore and GPU Architectures",
  * SIGMOD'17).  Citations "Lnnn" are lines of the paper transcript.
  *
- * What is computed (Def. 1-3, L86-105):
- *   Input P: n points over d dimensions, float32, smaller is better (footnote 2, L109).
- *   For every subspace 0 < delta < 2^d (bit i of delta <=> dimension i, L71), the subspace skyline
+ * What is computed (Def. 1-3, L92-110):
+ *   Input P: n points over d dimensions, float32, smaller is better (footnote 2, L114).
+ *   For every subspace 0 < delta < 2^d (bit i of delta <=> dimension i, L76), the subspace skyline
  *     S_delta(P) = { p : no q in P dominates p in delta }, where q dominates p in delta iff
  *     (B_{q=p} & delta) != delta and (B_{q<=p} & delta) == delta (Def. 1).
  *   The skycube (Def. 3) is returned in two forms:
- *     - per point, its membership bitmap (the paper's B_{p in S}, L79, here UNSHIFTED: bit delta, not
+ *     - per point, its membership bitmap (the paper's B_{p in S}, L84, here UNSHIFTED: bit delta, not
  *       bit delta-1);
- *     - per subspace, the ascending id list of S_delta(P) (the lattice of Fig. 1a, L151).
- *   Method: Alg. 3 (MDMC, L313-319) on the GPU: S+(P) prefilter (line 2), then one data-parallel task
+ *     - per subspace, the ascending id list of S_delta(P) (the lattice of Fig. 1a, L156).
+ *   Method: Alg. 3 (MDMC, L318-324) on the GPU: S+(P) prefilter (line 2), then one data-parallel task
  *   per p in S+(P) computing B_{p notin S} and B_{p notin S+} (lines 3-12), then compaction.
  *
  * Value semantics (readings Q9-Q12): IEEE binary32 compares only; -0 == +0; +-inf are
  * ordinary values; NaN is rejected (SKYCUBE_ENAN); equal points never dominate each other; ids are
- * the row indices of `points` (footnote 1, L73).
+ * the row indices of `points` (footnote 1, L78).
  *
  * Errors: every entry point returns a skycube_status; on any error the output struct is zeroed and
  * owns nothing; skycube_last_error() gives a thread-local detail string.  All calls are serialised
@@ -53,7 +53,7 @@ typedef struct {
     int32_t *ext_ids;          /* [n_ext] ascending ids of S+(P) */
     uint32_t words_per_row;    /* W = max(1, 2^d / 32) */
     uint32_t *membership;      /* [n * W] row p, bit delta (word delta>>5, bit delta&31) <=> p in S_delta(P);
-                                  bit 0 always 0; rows of points outside S+(P) are all zero (L101) */
+                                  bit 0 always 0; rows of points outside S+(P) are all zero (L106) */
     uint32_t *ext_membership;  /* [n * W] or NULL: bit delta <=> p in S+_delta(P) (SKYCUBE_EXT_MEMBERSHIP) */
     int64_t *cuboid_offsets;   /* [2^d + 1] or NULL (NO_LISTS): ids of S_delta are
                                   cuboid_ids[off[delta] .. off[delta+1]); off[0] = off[1] = 0 */
@@ -71,7 +71,7 @@ typedef struct {
                              only the subspaces with |delta| <= d' are computed and reported -- membership
                              bits of every delta with |delta| > d' are 0 and their lists are empty
                              (reading P1: "no correctness guarantee is offered for the skyline
-                             of said delta", L1180) */
+                             of said delta", L1248) */
 } skycube_opts;
 
 typedef struct {
@@ -81,6 +81,10 @@ typedef struct {
     int64_t pairs;         /* n_ext * (n_ext - 1): ordered S+ pairs tested by MDMC */
     int64_t total_ids;     /* sum over delta of |S_delta(P)| */
     int32_t kernel_launches;
+    double ms_comm;        /* multi-GPU exchange (flag and row gathers), host clock; 0 on one GPU */
+    int64_t exact_dts;     /* pairs that reached the exact dominance test of Alg. 3 line 10 (K3 misses) */
+    int64_t expansions;    /* contributing competitors expanded into the state (Alg. 3 lines 11-12) */
+    int32_t num_gpus;      /* devices the build ran on */
 } skycube_stats;
 
 /* Build the skycube of the host array points[n*d] (row-major, row = id, column i = dimension i).
@@ -108,7 +112,7 @@ skycube_status skycube_build_sdsc(const float *points, int64_t n, int32_t d, con
 /* ------------------------------------------------------------------------------------------------
  * HashCube output (Alg. 3 lines 1 and 13, L320; Appendix B.1; Fig. 1b).
  * Point p is represented by B_{p notin S}: 2^d - 1 bits, bit delta-1 set <=> p is dominated in delta
- * (the shifted order of L79).  It is cut into n_words = ceil((2^d - 1) / w) words of w bits (word k =
+ * (the shifted order of L84).  It is cut into n_words = ceil((2^d - 1) / w) words of w bits (word k =
  * subspaces k*w+1 .. k*w+w; the last word may be shorter) and word k is hashed by h_k: key = the word's
  * value, value = the ids of the points with that key.  A point whose word is all set (dominated in all
  * of the word's subspaces) is not stored (L1278); points outside S+(P) are never stored.
@@ -150,6 +154,13 @@ skycube_status skycube_hashcube_query(const skycube_hashcube *hc, uint32_t delta
 
 const char *skycube_strerror(skycube_status s);
 const char *skycube_last_error(void);   /* thread-local detail of the last error */
+
+/* Process-wide tuning / test overrides (performance only: every setting gives the same output bytes).
+ * Keys: "k3_design" ('A', 'O' or 0 = automatic), "k3_tpc" (K3 tasks per CTA, 0 = automatic), "k3_mode"
+ * (K3 state mode 0/1/2, -1 = automatic), "share_devices" (1: num_gpus ranks may share devices, so the
+ * multi-GPU logic can be tested on one GPU), "reset" (all automatic).  EINVAL for an unknown key or value.
+ * Serialised with the build calls. */
+skycube_status skycube_set_tuning(const char *key, int32_t value);
 
 /* ------------------------------------------------------------------------------------------------
  * Device-resident entry points (used by the per-rank multi-GPU driver and the benchmark).

@@ -4,7 +4,7 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py`` (its ``cpu_baselin
 ``--impl reference``) may import this package.  The product path
 (``paper_conf_sigmod_boghcsa17_b200``) never imports it and shares no code with it.
 
-The arithmetic lives in ``skycube_oracle.c`` (Def. 1-3 of PAPER.md L86-105, written out; see the
+The arithmetic lives in ``skycube_oracle.c`` (Def. 1-3 of PAPER.md L92-110, written out; see the
 header of that file).  This module only compiles it with gcc and marshals numpy arrays.
 
 Functions
@@ -12,7 +12,7 @@ Functions
 rows_a(x)            Oracle A (literal per-subspace definition): (membership rows, extended rows)
 rows_b(x, pids)      Oracle B (per point, all of P, superset closures)
 cells_a(x, p, delta) Oracle A on individual (point, subspace) cells
-ext_full(x)          S+(P), Alg. 3 line 2 (L315)
+ext_full(x)          S+(P), Alg. 3 line 2 (L320)
 lattice(rows, d)     CSR lattice (Fig. 1a) from rows: offsets[2^d+1], ids ascending per subspace
 
 Parity status: every function is pinned by tests/test_oracle_*.py (no "parity unpinned" entries).
@@ -34,13 +34,21 @@ _lib = None
 
 
 def build(force: bool = False) -> str:
-    """Compile the oracle with gcc -O2 -fopenmp (plain C, no GPU)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+    """Compile the oracle with gcc -O2 -fopenmp (plain C, no GPU).
+
+    ``SKYCUBE_ORACLE_CFLAGS`` (space-separated) replaces ``-O2`` and builds a separately named
+    library; ``tools/oracle_digest.py`` uses ``-O3 -march=native -funroll-loops`` for its multi-hour
+    full-size runs.  The source, and so the arithmetic, is the same (no -ffast-math: the oracle's only
+    operations on values are IEEE ``<`` / ``<=``).  Timed baselines (bench.py) use the default."""
+    flags = os.environ.get("SKYCUBE_ORACLE_CFLAGS", "").split() or ["-O2"]
+    lib = _LIB if flags == ["-O2"] else _LIB.replace(
+        ".so", "_" + "".join(c for c in "".join(flags) if c.isalnum()) + ".so")
+    if force or not os.path.exists(lib) or os.path.getmtime(lib) < os.path.getmtime(_SRC):
+        tmp = lib + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *flags, "-fopenmp", "-fPIC", "-shared", "-std=c11",
                                "-o", tmp, _SRC])
-        os.replace(tmp, _LIB)
-    return _LIB
+        os.replace(tmp, lib)
+    return lib
 
 
 def _load():

@@ -7,23 +7,23 @@
  *
  * It is plain, slow and written to be checked against PAPER.md by eye:
  *
- *   Def. 1 (L86-88, §2.2): p dominates q in subspace 0 < delta < 2^d  iff
+ *   Def. 1 (L92, §2.2): p dominates q in subspace 0 < delta < 2^d  iff
  *        (B_{p=q} & delta) != delta  and  (B_{p<=q} & delta) == delta;
  *        p strictly dominates q in delta iff additionally (B_{p=q} & delta) == 0.
- *   Def. 2 (L95-97): S_delta(P)  = { q in P : no p in P with p dominates q in delta }
+ *   Def. 2 (L100): S_delta(P)  = { q in P : no p in P with p dominates q in delta }
  *                    S+_delta(P) = { q in P : no p in P with p strictly dominates q in delta }
- *   Def. 3 (L105):   the skycube maps every 0 < delta < 2^d to S_delta(P).
- *   Bitmasks (L71-79, §2.1): bit i of delta <=> dimension i; bit i of B_{p (op) q} <=> p[i] (op) q[i].
- *   Smaller values are better (footnote 2, L109).  Values are IEEE binary32 compared with < and <=
+ *   Def. 3 (L110):   the skycube maps every 0 < delta < 2^d to S_delta(P).
+ *   Bitmasks (L76-84, §2.1): bit i of delta <=> dimension i; bit i of B_{p (op) q} <=> p[i] (op) q[i].
+ *   Smaller values are better (footnote 2, L114).  Values are IEEE binary32 compared with < and <=
  *   (reading Q10); no arithmetic is applied to them.
  *
  * Output conventions: membership row of point p = W = max(1, 2^d/32) uint32
  * words; bit delta (word delta>>5, bit delta&31) set <=> p in S_delta(P); bit 0 is always 0.
- * This is the paper's B_{p in S} (L79) unshifted (the paper stores bit delta-1).
+ * This is the paper's B_{p in S} (L84) unshifted (the paper stores bit delta-1).
  *
  * Two independent algorithms:
  *   oracle_a_*  literal Def. 1-3: per subspace, per point, per competitor (O(2^d n^2 d)).
- *   oracle_b_*  per point p against all of P (not only S+; it does not use the S+ lemma of L101):
+ *   oracle_b_*  per point p against all of P (not only S+; it does not use the S+ lemma of L106):
  *               p is dominated in delta  <=>  exists q, exists i in delta:  i in S_qp  and  delta is a
  *               subset of L_qp, where L_qp = B_{q<=p}, S_qp = B_{q<p}.  With G_i = { L_qp : i in S_qp }
  *               and D_i = superset-closure(G_i) (D_i[delta] = OR_{M superset of delta} G_i[M]),
@@ -44,7 +44,7 @@ static inline uint32_t words_per_row(int d) {
     return d >= 5 ? (1u << (d - 5)) : 1u;
 }
 
-/* B_{q<=p} and B_{q<p} (L77: bit i of B_{p (op) q} is set iff p[i] (op) q[i]). */
+/* B_{q<=p} and B_{q<p} (L82: bit i of B_{p (op) q} is set iff p[i] (op) q[i]). */
 static inline void relation_masks(const float *q, const float *p, int d, uint32_t *le, uint32_t *lt) {
     uint32_t a = 0, b = 0;
     for (int i = 0; i < d; i++) {
@@ -97,7 +97,7 @@ int oracle_a_rows(const float *pts, int64_t n, int d, uint32_t *rows, uint32_t *
         for (uint32_t delta = 1; delta <= full; delta++) {
             int dominated = 0, sdominated = 0;
             for (int64_t q = 0; q < n; q++) {
-                if (q == p) continue;                          /* "a distinct point" (L83) */
+                if (q == p) continue;                          /* "a distinct point" (L88) */
                 const float *qq = pts + (size_t)q * d;
                 if (!dominated && dominates(qq, pp, d, delta)) dominated = 1;
                 if (!sdominated && strictly_dominates(qq, pp, d, delta)) sdominated = 1;
@@ -130,7 +130,7 @@ int oracle_a_cells(const float *pts, int64_t n, int d, const int64_t *pids, cons
     return 0;
 }
 
-/* S+(P) of Alg. 3 line 2 (L315): ext[p] = 1 iff no q strictly dominates p in the full space. */
+/* S+(P) of Alg. 3 line 2 (L320): ext[p] = 1 iff no q strictly dominates p in the full space. */
 int oracle_ext_full(const float *pts, int64_t n, int d, uint8_t *ext) {
     if (d < 1 || d > 16) return 1;
     const uint32_t full = (1u << d) - 1u;
@@ -211,7 +211,7 @@ int oracle_b_rows(const float *pts, int64_t n, int d, const int64_t *pids, int64
 }
 
 /* ---------------------------------------------------------------------------------------------
- * Lattice (Fig. 1a, L151: "for each subspace delta, a flat array stores the point ids of S_delta")
+ * Lattice (Fig. 1a, L156: "for each subspace delta, a flat array stores the point ids of S_delta")
  * from membership rows: offsets[2^d + 1], ids ascending within each delta (reading Q12).
  * Call once with ids == NULL to get offsets (total = offsets[2^d]), then again with ids.
  * ------------------------------------------------------------------------------------------- */

@@ -26,6 +26,7 @@ EXPORTED = (
     "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
     "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_free",
     "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc",
+    "skycube_set_tuning",
 )
 
 
@@ -67,7 +68,8 @@ class Stats(ctypes.Structure):
     _fields_ = [(k, ctypes.c_double) for k in ("ms_total", "ms_h2d", "ms_validate", "ms_sort", "ms_codes",
                                                 "ms_prefilter", "ms_mdmc", "ms_compact", "ms_d2h")] + [
         ("n_ext", ctypes.c_int64), ("pairs", ctypes.c_int64), ("total_ids", ctypes.c_int64),
-        ("kernel_launches", ctypes.c_int32)]
+        ("kernel_launches", ctypes.c_int32), ("ms_comm", ctypes.c_double), ("exact_dts", ctypes.c_int64),
+        ("expansions", ctypes.c_int64), ("num_gpus", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -114,13 +116,29 @@ def lib():
         L.skycube_ctx_set_max_level.argtypes = [P, I32]
         L.skycube_dev_hashcube.argtypes = [P, P, U32, P, P, P, P, ctypes.POINTER(I64), ctypes.POINTER(I64),
                                            ctypes.POINTER(I64), P]
-        for f in ("skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
+        L.skycube_set_tuning.argtypes = [ctypes.c_char_p, I32]
+        for f in ("skycube_set_tuning", "skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
                   "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_query",
                   "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
+        # tools/*.sh A/B runs name tuning overrides in the environment; applied once, here, never in the
+        # library's launch path
+        for key, env in (("k3_design", "SKYCUBE_K3_DESIGN"), ("k3_tpc", "SKYCUBE_K3_TPC"),
+                         ("k3_mode", "SKYCUBE_K3_MODE"), ("share_devices", "SKYCUBE_SHARE_DEVICES")):
+            v = os.environ.get(env, "")
+            if v:
+                set_tuning(key, ord(v[0]) if key == "k3_design" else int(v))
     return _lib
+
+
+def set_tuning(key: str, value: int) -> None:
+    """skycube_set_tuning: performance-only overrides (k3_design 'A'/'O' as ord(), k3_tpc, k3_mode,
+    share_devices) or key "reset"."""
+    if isinstance(value, str):
+        value = ord(value[0])
+    _check(lib().skycube_set_tuning(key.encode(), int(value)))
 
 
 def _check(status):
@@ -389,7 +407,7 @@ class Context:
         a = np.zeros(8, np.int64)
         _check(lib().skycube_ctx_counters(self._h, a.ctypes.data_as(ctypes.c_void_p)))
         return {"k1_box": int(a[0]), "k1_pair": int(a[1]), "k3_box": int(a[2]), "k3_pair": int(a[3]),
-                "k3_miss": int(a[4]), "k3_sub": int(a[5])}
+                "k3_miss": int(a[4]), "k3_sub": int(a[5]), "k3_expansions": int(a[6])}
 
     def info(self):
         m, W, ex = ctypes.c_int64(), ctypes.c_uint32(), ctypes.c_uint32()

@@ -20,6 +20,13 @@ struct skycube_ctx {
     cudaEvent_t ev_ext = nullptr, ev_side = nullptr;
 };
 
+namespace sky {
+Tuning &tuning() {
+    static Tuning t;
+    return t;
+}
+}  // namespace sky
+
 namespace {
 
 std::mutex g_mutex;                  // serialises skycube_build* (header: "calls are serialised")
@@ -133,6 +140,21 @@ skycube_status guarded(F &&f) {
     }
 }
 
+// K3 work counters (exact DTs = misses, expansions) of a context, for skycube_stats
+void read_k3_counters(const sky::Ctx &c, int64_t *exact_dts, int64_t *expansions) {
+    int64_t a[8] = {0};
+    SKY_CUDA(cudaMemcpy(a, c.counters.p, sizeof(a), cudaMemcpyDeviceToHost));
+    *exact_dts = a[4];
+    *expansions = a[6];
+}
+
+// Failure after kernels may have been queued: wait for every stream of the device before the result's
+// pinned buffers go back to the pool (K3 writes the membership rows straight into one of them).
+void drain_device(int device) {
+    if (cudaSetDevice(device) == cudaSuccess) cudaDeviceSynchronize();
+    cudaGetLastError();
+}
+
 float ev_ms(cudaEvent_t a, cudaEvent_t b) {
     float ms = 0.f;
     cudaEventElapsedTime(&ms, a, b);
@@ -209,8 +231,7 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
             cudaGetLastError();
             throw sky::Error{SKYCUBE_ENODEV, "no CUDA device visible"};
         }
-        const char *share_env = getenv("SKYCUBE_SHARE_DEVICES");
-        const bool share = share_env && share_env[0] == '1';
+        const bool share = sky::tuning().share_devices == 1;
         if (!share && first + k > count)
             throw sky::Error{SKYCUBE_ENODEV, "num_gpus exceeds the visible devices after `device`"};
         std::vector<int> dev(k);
@@ -333,9 +354,13 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
             int64_t launches = 0;
             for (int g = 0; g < k; g++) launches += xs[g]->c.L.count;
             stats->kernel_launches = (int32_t)(launches - launches0);
+            stats->num_gpus = k;
         }
     });
     if (st != SKYCUBE_OK) {
+        int count = 0;
+        if (cudaGetDeviceCount(&count) != cudaSuccess) count = 0;
+        for (int g = 0; g < k && count > 0; g++) drain_device((first + g) % count);
         skycube_free(&r);
         return st;
     }
@@ -363,6 +388,30 @@ const char *skycube_strerror(skycube_status s) {
 }
 
 const char *skycube_last_error(void) { return g_last_error.c_str(); }
+
+skycube_status skycube_set_tuning(const char *key, int32_t value) {
+    if (!key) return fail(SKYCUBE_EINVAL, "key == NULL");
+    std::lock_guard<std::mutex> lk(g_mutex);
+    sky::Tuning &t = sky::tuning();
+    const std::string k(key);
+    if (k == "k3_design") {
+        if (value != 0 && value != 'A' && value != 'O') return fail(SKYCUBE_EINVAL, "k3_design must be 0, 'A' or 'O'");
+        t.k3_design = value;
+    } else if (k == "k3_tpc") {
+        if (value < 0) return fail(SKYCUBE_EINVAL, "k3_tpc must be >= 0");
+        t.k3_tpc = value;
+    } else if (k == "k3_mode") {
+        if (value < -1 || value > 2) return fail(SKYCUBE_EINVAL, "k3_mode must be in [-1, 2]");
+        t.k3_mode = value;
+    } else if (k == "share_devices") {
+        t.share_devices = value ? 1 : 0;
+    } else if (k == "reset") {
+        t = sky::Tuning();
+    } else {
+        return fail(SKYCUBE_EINVAL, "unknown tuning key " + k);
+    }
+    return SKYCUBE_OK;
+}
 
 void skycube_free(skycube_result *out) {
     if (!out) return;
@@ -407,6 +456,8 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
         else check_device(device);
         sky::Ctx &c = x->c;
         const int64_t launches0 = c.L.count;
+        int64_t dts0 = 0, exp0 = 0;
+        if (stats) read_k3_counters(c, &dts0, &exp0);
         const bool want_ext = (flags & SKYCUBE_EXT_MEMBERSHIP) != 0;
         if (n == 0) {
             if (!(flags & SKYCUBE_NO_LISTS)) {
@@ -477,9 +528,14 @@ skycube_status skycube_build_ex(const float *points, int64_t n, int32_t d, const
             stats->pairs = m * (m > 0 ? m - 1 : 0);
             stats->total_ids = total;
             stats->kernel_launches = (int32_t)(c.L.count - launches0);
+            read_k3_counters(c, &stats->exact_dts, &stats->expansions);
+            stats->exact_dts -= dts0;
+            stats->expansions -= exp0;
+            stats->num_gpus = 1;
         }
     });
     if (st != SKYCUBE_OK) {
+        drain_device(device);
         skycube_free(&r);
         return st;
     }
@@ -566,11 +622,14 @@ skycube_status skycube_build_sdsc(const float *points, int64_t n, int32_t d, con
         }
     });
     if (st != SKYCUBE_OK) {
+        drain_device(device);
         skycube_free(&r);
         return st;
     }
-    if (stats)
+    if (stats) {
+        stats->num_gpus = 1;
         stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    }
     *out = r;
     return SKYCUBE_OK;
 }
@@ -653,9 +712,11 @@ skycube_status skycube_build_hashcube(const float *points, int64_t n, int32_t d,
         }
     });
     if (st != SKYCUBE_OK) {
+        drain_device(device);
         skycube_hashcube_free(&r);
         return st;
     }
+    if (stats) stats->num_gpus = 1;
     if (stats)
         stats->ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     *out = r;

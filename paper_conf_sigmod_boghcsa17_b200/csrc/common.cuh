@@ -40,6 +40,16 @@ struct Error {
             throw ::sky::Error{4, std::string("kernel launch: ") + cudaGetErrorString(_e)};     \
     } while (0)
 
+// Process-wide tuning / test overrides (skycube_set_tuning in the C-ABI; never read from the environment in
+// the launch path).  0 = automatic.
+struct Tuning {
+    int k3_design = 0;      // 'A' or 'O': force a K3 design
+    int k3_tpc = 0;         // force K3 tasks per CTA (design A)
+    int k3_mode = -1;       // force a K3 state mode (0, 1, 2); -1 = automatic
+    int share_devices = 0;  // 1: multi-GPU ranks may share devices (tests of the k-rank logic on one GPU)
+};
+Tuning &tuning();
+
 inline uint32_t words_per_row(int d) { return d >= 5 ? (1u << (d - 5)) : 1u; }
 inline int dpad_of(int d) { return ((d + 3) / 4) * 4; }  // codes padded to groups of 4 dims
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }

@@ -1,4 +1,4 @@
-// k1_prefilter.cu — K1: the extended skyline S+(P) of Alg. 3 line 2 (L315).
+// k1_prefilter.cu — K1: the extended skyline S+(P) of Alg. 3 line 2 (L320).
 //
 //   p in S+(P)  <=>  no q in P strictly dominates p in the full space (Def. 1-2, delta = 2^d - 1).
 //

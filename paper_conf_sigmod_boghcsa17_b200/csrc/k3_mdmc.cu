@@ -1,7 +1,7 @@
-// k3_mdmc.cu — K3: the MDMC per-point task of Alg. 3 (L313-319), lines 3-12, on sm_100a.
+// k3_mdmc.cu — K3: the MDMC per-point task of Alg. 3 (L318-324), lines 3-12, on sm_100a.
 //
-// For every p in S+(P) (the data-parallel tasks, L306-310) and every competitor q in S+(P) (Λ1:
-// competitors outside S+ add nothing), the pair reduces to two d-bit masks (L77)
+// For every p in S+(P) (the data-parallel tasks, L308-310) and every competitor q in S+(P) (Λ1:
+// competitors outside S+ add nothing), the pair reduces to two d-bit masks (L82)
 //     L = B_{q<=p},  S = B_{q<p}   (E = L \ S = B_{q=p})
 // and q dominates p exactly in the subspaces { delta subset of L : delta & S != 0 } (Def. 1), strictly in the
 // non-empty subsets of S.  B_{p notin S+} (strict) is downward closed, so bit L set in it means q adds
@@ -10,7 +10,7 @@
 // Competitors are S+ in static-tree (Morton) order, in chunks of 32 with their lower corner, visited
 // strongest corner first (prep.cu).  For a task p and a chunk, Mbox = B_{corner<=p} is a superset of M(q,p)
 // for every q of the chunk, so bit Mbox set in the probe set proves the whole chunk adds nothing (Λ4 on a
-// leaf range: the paper's filter on path labels, L320-328, with the tree's global pivots).
+// leaf range: the paper's filter on path labels, L446-452, with the tree's global pivots).
 //
 // Design A (k3_mdmc_kernel): a CTA holds up to NT tasks (codes + state in shared memory) and streams every
 // chunk once (TMA ring fed by one producer warp); each of the 16 consumer warps takes one chunk per tile, one
@@ -45,7 +45,6 @@
 // The result is scheduling-independent (every update is an OR of a correct contribution, every skip is
 // sound for any subset of the final state), so racing warps and any chunk order give identical bytes.
 #include <algorithm>
-#include <cstdlib>
 
 #include "ctx.cuh"
 #include "tile_stream.cuh"
@@ -375,7 +374,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         return;
     }
     const int ngroups = (nt + 31) >> 5;
-    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0;
+    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t *rec = ring.stage(tile) + warp * REC;
@@ -421,6 +420,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
                 if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
             }
             uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
+            n_exp += __popc(todo);
             while (todo) {
                 const int from = __ffs(todo) - 1;
                 todo &= todo - 1;
@@ -521,6 +521,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         if (lane == 0) {
             atomicAdd(&counters[4], n_miss);
             atomicAdd(&counters[5], n_sub);
+            atomicAdd(&counters[6], n_exp);
         }
     }
     consumer_sync(kWarps * 32);
@@ -607,7 +608,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     uint32_t p[G::CW];
     load_row_s<G::CW>(pV_s + 4u * (town * CWV), p);
     const uint32_t st_own = st_s + 4u * (town * C::PS);
-    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0;
+    unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t stg_s = ring_s + 4u * (uint32_t)(tile % kStages) * (uint32_t)C::TW;
@@ -636,6 +637,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
                 if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
             }
             uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
+            n_exp += __popc(todo);
             while (todo) {
                 const int from = __ffs(todo) - 1;
                 todo &= todo - 1;
@@ -730,6 +732,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
             atomicAdd(&counters[3], n_pair);
             atomicAdd(&counters[4], n_miss);
             atomicAdd(&counters[5], n_sub);
+            atomicAdd(&counters[6], n_exp);
         }
     }
     consumer_sync(kWarps * 32);
@@ -780,9 +783,9 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     using C = GeoK3<D, MODE>;
     static_assert(C::NT >= 1, "shared memory too small for one task per CTA");
     // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
-    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  SKYCUBE_K3_DESIGN=A|O forces one.
-    const char *design = getenv("SKYCUBE_K3_DESIGN");
-    const bool want_o = design && *design ? design[0] == 'O' : MODE == kModeDims;
+    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
+    const int design = tuning().k3_design;
+    const bool want_o = design ? design == 'O' : MODE == kModeDims;
     if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
@@ -799,7 +802,7 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
                 tpc = t;
             }
     }
-    if (const char *e = getenv("SKYCUBE_K3_TPC"); e && *e) tpc = std::max(1, std::min<int>(C::NT, atoi(e)));
+    if (tuning().k3_tpc > 0) tpc = std::max(1, std::min<int>(C::NT, tuning().k3_tpc));
     const size_t smem = C::smem_bytes(tpc);
     SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
@@ -814,16 +817,15 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
 
 // Tie-heavy inputs (every dimension discrete enough for injective codes) or d <= 10: the tie-exact state
 // (kModeDims, d <= 12) unless B_{p notin S+} itself is requested (ext rows), then kModeSmemTie.  Continuous
-// data at d > 10: ties are rare and go to a global row (kModeGlobalTie).  SKYCUBE_K3_MODE=0|1|2 forces a
-// mode (parity tests of every mode on the same inputs).
+// data at d > 10: ties are rare and go to a global row (kModeGlobalTie).  skycube_set_tuning("k3_mode", m)
+// forces a mode (parity tests of every mode on the same inputs).
 template <int D>
 void launch(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
             cudaStream_t st) {
     const bool all_exact = c.exact_mask == ((1u << D) - 1u);
-    const char *m = getenv("SKYCUBE_K3_MODE");
     int mode = (D <= 10 || all_exact) ? (D <= 12 && !ext_rows32 ? kModeDims : kModeSmemTie) : kModeGlobalTie;
-    if (m && *m) {
-        mode = m[0] - '0';
+    if (tuning().k3_mode >= 0) {
+        mode = tuning().k3_mode;
         if (mode == kModeDims && (D > 12 || ext_rows32)) mode = kModeSmemTie;
     }
     if (mode == kModeDims) {

@@ -1,5 +1,5 @@
 // k4_compact.cu — K4: from the per-point membership rows (complement of B_{p notin S}, Alg. 3 line 13)
-// to (a) the row-major membership bitmap by point id and (b) the lattice of Fig. 1a (L151): for every
+// to (a) the row-major membership bitmap by point id and (b) the lattice of Fig. 1a (L156): for every
 // subspace delta the ascending id list of S_delta(P).
 //
 // Input: rows of the S+ points in the tiled layout of K3: group g of 32 consecutive S+ points (id
@@ -43,7 +43,7 @@ __global__ void membership_kernel(const uint32_t *__restrict__ rows32, const int
     }
 }
 
-// Zero the rows of the points outside S+ (L101: they are in no skyline); one thread per word.
+// Zero the rows of the points outside S+ (L106: they are in no skyline); one thread per word.
 __global__ void zero_outside_kernel(const uint32_t *__restrict__ ext_id_flag, int64_t n, uint32_t W,
                                     uint32_t *__restrict__ membership) {
     const int64_t total = n * (int64_t)W;

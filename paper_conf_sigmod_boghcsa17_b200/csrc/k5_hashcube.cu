@@ -1,9 +1,9 @@
 // k5_hashcube.cu — K5: the HashCube output of MDMC (Alg. 3 lines 1 and 13, L320; Appendix B.1,
 // L1274-1282; Fig. 1b).  Each point p is represented by B_{p notin S} (2^d - 1 bits, bit delta-1 <=> p is
-// dominated in delta, the shifted order of L79); the bitmask is cut into words of w bits and word k is
+// dominated in delta, the shifted order of L84); the bitmask is cut into words of w bits and word k is
 // hashed by h_k: key = the word, value = the ids of the points with that word.  A point whose word is
 // all set (dominated in all w subspaces) is not stored (L1278).  Points outside S+(P) are dominated
-// everywhere (L101) and never stored, so only the S+ rows of K3 are read.
+// everywhere (L106) and never stored, so only the S+ rows of K3 are read.
 //
 // The hash maps are materialised as sorted arrays (reading H1): for every word k its distinct
 // keys ascending, each with its ascending id list.  GPU construction, all HBM-bound:

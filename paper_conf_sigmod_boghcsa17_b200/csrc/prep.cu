@@ -1,7 +1,7 @@
 // prep.cu — K0 (validate + canonicalise + order-preserving keys), the key-sum order of Λ2, and
 // K2 (per-dimension monotone 15-bit codes), plus the S+ gathers after the prefilter.
 //
-// Paper: Alg. 3 line 2 (L315) builds "quad tree T over S+(P)" with global pivots (median, quartiles,
+// Paper: Alg. 3 line 2 (L320) builds "quad tree T over S+(P)" with global pivots (median, quartiles,
 // octiles: L338, L348-356; Fig. 3): every point gets, per dimension, its bin among
 // statically defined global thresholds, and two points are compared through their bins (Eq. 1,
 // L1312) before any exact dominance test.  This repo keeps that idea — global, monotone,
@@ -153,12 +153,16 @@ __global__ void k2_pad_kernel(int64_t n, int d, int dp, uint16_t *__restrict__ c
 }
 
 __global__ void gather_sorted_kernel(const uint32_t *__restrict__ perm, const uint32_t *__restrict__ codes_id,
-                                     const uint32_t *__restrict__ ord, int64_t n, int d, int cw,
+                                     const uint32_t *__restrict__ ord, int64_t n, int64_t npad, int d, int cw,
                                      uint32_t *__restrict__ codes_sorted, uint32_t *__restrict__ ord_sorted) {
     const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (s >= n) {  // padding up to whole chunks: codes that are never better than a task
+    if (s >= n) {  // padding up to whole chunk tiles: codes and exact keys that are never better than a task
         if (s < ((n + 31) / 32) * 32)
             for (int k = 0; k < cw; k++) codes_sorted[s * cw + k] = 0x7fff7fffu;
+        // K1's tie path reads the exact keys of every competitor slot of a chunk it opens, padding included
+        // (a task with code 0x7fff in every inexact dimension ties the padding codes there)
+        if (s < npad)
+            for (int i = 0; i < d; i++) ord_sorted[s * d + i] = 0xffffffffu;
         return;
     }
     const int64_t id = perm[s];
@@ -287,7 +291,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.nanflag.ensure(sizeof(uint32_t));
     c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
     c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
-    c.ord_sorted.ensure(sizeof(uint32_t) * nd);
+    c.ord_sorted.ensure(sizeof(uint32_t) * npad * d);
     c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * kRecAll * cw);
 
     SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
@@ -331,7 +335,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     radix_sort_u64(c.keysum.as<uint64_t>(), c.perm.as<uint32_t>(), n, bits_per_dim * d, c.keys_alt.as<uint64_t>(),
                    c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
     gather_sorted_kernel<<<blocks_for(npad, 256), 256, 0, st>>>(c.perm.as<uint32_t>(), c.codes_id.as<uint32_t>(),
-                                                               c.ord.as<uint32_t>(), n, d, cw,
+                                                               c.ord.as<uint32_t>(), n, npad, d, cw,
                                                                c.codes_sorted.as<uint32_t>(), c.ord_sorted.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();

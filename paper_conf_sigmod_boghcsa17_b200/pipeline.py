@@ -1,6 +1,6 @@
 """Per-rank device pipeline of the MDMC skycube, one process per GPU (torch.distributed for plumbing).
 
-Sharding (the paper's device-level data parallelism of MDMC, L306-310, L420 "every
+Sharding (the paper's device-level data parallelism of MDMC, L308-310, L420 "every
 task is independent, there is no need for synchronisation"):
 
   1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic)

@@ -34,7 +34,7 @@ def fig3_string(rows, p, d, negate):
 
 
 def shifted_string(rows, p, d):
-    """The paper's B_{p in S} (L79): bit delta-1, most significant (delta = 2^d - 1) first."""
+    """The paper's B_{p in S} (L84): bit delta-1, most significant (delta = 2^d - 1) first."""
     return "".join("1" if bit(rows, p, delta) else "0" for delta in range((1 << d) - 1, 0, -1))
 
 

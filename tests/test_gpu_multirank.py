@@ -82,9 +82,9 @@ def test_multirank_bytes_equal_single_rank(world, name):
 
 
 @pytest.mark.parametrize("k,name", [(2, "C3I"), (3, "A-small"), (4, "ct-small"), (2, "C2")])
-def test_capi_num_gpus_bytes_equal_single_gpu(monkeypatch, k, name):
+def test_capi_num_gpus_bytes_equal_single_gpu(tuning, k, name):
     """The C-ABI's single-process multi-GPU path (skycube_opts.num_gpus = k): k logical ranks, here sharing
-    the one GPU (SKYCUBE_SHARE_DEVICES=1), with the flag OR-combine, the peer-copy gathers and the sharded
+    the one GPU (skycube_set_tuning("share_devices", 1)), with the flag OR-combine, the peer-copy gathers and the sharded
     K1/K3 ranges; every output byte must equal the one-GPU build."""
     import torch
     import paper_conf_sigmod_boghcsa17_b200 as sky
@@ -97,7 +97,7 @@ def test_capi_num_gpus_bytes_equal_single_gpu(monkeypatch, k, name):
     else:
         x = datagen.config(name).data()
     want = sky.skycube_build(x)
-    monkeypatch.setenv("SKYCUBE_SHARE_DEVICES", "1")
+    tuning("share_devices", 1)
     with sky.skycube_build_raw(x, num_gpus=k, stats=True) as r:
         assert np.array_equal(r.membership(), want["rows"])
         assert np.array_equal(r.ext_ids(), want["ext_ids"])

@@ -124,6 +124,28 @@ def test_inexact_codes_continuous(dist, d):
     assert np.array_equal(r["rows"][pids], oracle.rows_b(x, pids))
 
 
+def test_k1_padding_keys_all_inexact_max_code():
+    # K1's tie path reads the exact keys of the padding competitors of the last chunk.  Every
+    # dimension inexact (> 2^15 distinct values), p = (MAX, MAX) holding code 0x7fff everywhere, n not a
+    # multiple of 32: the padding codes tie p in every dimension, so only their exact keys (never better)
+    # keep p in S+.  A larger build first leaves other keys in the reused buffers.
+    sky.skycube_build(datagen.generate("I", 120_000, 2, 9))
+    h = 33_000
+    rng = np.random.default_rng(11)
+    xs = rng.permutation(h).astype(np.float32)
+    big = np.float32(1e6)
+    x = np.concatenate([np.stack([xs, np.full(h, big, np.float32)], 1),
+                        np.stack([np.full(h, big, np.float32), xs], 1),
+                        np.array([[big, big]], np.float32)])
+    x = np.ascontiguousarray(x[rng.permutation(x.shape[0])])
+    assert x.shape[0] % 32 != 0
+    r = gpu(x)
+    assert np.array_equal(r["ext_ids"], np.nonzero(oracle.ext_full(x))[0])
+    pmax = int(np.nonzero((x[:, 0] == big) & (x[:, 1] == big))[0][0])
+    pids = np.concatenate([[pmax], rng.choice(x.shape[0], 40, replace=False)])
+    assert np.array_equal(r["rows"][pids], oracle.rows_b(x, pids))
+
+
 def test_edge_cases():
     # n = 1
     r = gpu(np.array([[0.5, 0.25, 0.75]], np.float32))
@@ -171,10 +193,10 @@ def test_row_permutation_invariance():
 
 @pytest.mark.parametrize("mode", ["0", "1", "2"])
 @pytest.mark.parametrize("d", [3, 6, 9, 11, 12])
-def test_k3_state_modes_tie_heavy(monkeypatch, mode, d):
+def test_k3_state_modes_tie_heavy(tuning, mode, d):
     """Every K3 state mode (global tie row / shared-memory tie row / per-dimension sets) on tie-heavy data,
     including values tied at each dimension's minimum (Z_p of the per-dimension mode)."""
-    monkeypatch.setenv("SKYCUBE_K3_MODE", mode)
+    tuning("k3_mode", int(mode))
     x = datagen.small_int_grid(700, d, 4, 300 + d)
     x[::7, d - 1] = x[:, d - 1].min()
     want = oracle.rows_b(x)
@@ -205,11 +227,11 @@ def test_repeat_builds_multi_tile_high_d(d):
 @pytest.mark.parametrize("design", ["A", "O"])
 @pytest.mark.parametrize("mode", ["0", "1", "2"])
 @pytest.mark.parametrize("case", [("A", 6000, 12, 901), ("I", 5000, 9, 902), ("A", 3000, 14, 903), ("C", 4000, 6, 904)])
-def test_k3_designs_and_modes(monkeypatch, design, mode, case):
+def test_k3_designs_and_modes(tuning, design, mode, case):
     """Both K3 designs (A: chunk-owner warps; O: task-owner warps, the default where 32 tasks' state fits in
     shared memory) under every state mode, on continuous data spanning many chunk tiles with ragged tails."""
-    monkeypatch.setenv("SKYCUBE_K3_DESIGN", design)
-    monkeypatch.setenv("SKYCUBE_K3_MODE", mode)
+    tuning("k3_design", design)
+    tuning("k3_mode", int(mode))
     dist, n, d, seed = case
     x = datagen.generate(dist, n, d, seed)
     want = oracle.rows_b(x)

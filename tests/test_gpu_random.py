@@ -44,16 +44,16 @@ def _dataset(rng):
 
 
 @pytest.mark.parametrize("seed", range(300))
-def test_random_case(monkeypatch, seed):
+def test_random_case(tuning, seed):
     rng = np.random.default_rng(10_000 + seed)
     x = _dataset(rng)
     n, d = x.shape
     design = ["", "A", "O"][int(rng.integers(0, 3))]
     mode = ["", "0", "1", "2"][int(rng.integers(0, 4))]
     if design:
-        monkeypatch.setenv("SKYCUBE_K3_DESIGN", design)
+        tuning("k3_design", design)
     if mode:
-        monkeypatch.setenv("SKYCUBE_K3_MODE", mode)
+        tuning("k3_mode", int(mode))
     want = oracle.rows_b(x)
     level = int(rng.integers(0, d + 1)) if rng.random() < 0.3 else 0
     r = sky.skycube_build(x, max_level=level)

@@ -34,7 +34,7 @@ def test_flights_minutes_same_skycube():
     assert (a == b).all()
 
 
-def test_flights_shifted_membership_L79():
+def test_flights_shifted_membership_L84():
     rows = oracle.rows_b(FLIGHTS)
     assert shifted_string(rows, 1, 3) == GOLD["shifted_in_S_f1"]
 
@@ -50,11 +50,11 @@ def test_flights_fig3_masks(method):
         assert fig3_string(ext, p, 3, negate=True) == GOLD["fig3_not_in_Sp"][p], p
 
 
-def test_flights_extended_skylines_L99():
+def test_flights_extended_skylines_L104():
     rows, ext = oracle.rows_a(FLIGHTS)
     assert members(rows, 3) == GOLD["S3"]
     assert members(ext, 3) == GOLD["Splus3"]
-    # L89-91: f3 strictly dominates f4 in 6 (f4 not in S+_6); f3 dominates f4 in 7 but not strictly
+    # L94-96: f3 strictly dominates f4 in 6 (f4 not in S+_6); f3 dominates f4 in 7 but not strictly
     assert not bit(ext, 4, 6) and not bit(rows, 4, 7) and bit(ext, 4, 7)
     # f1 dominates f0 in delta = 3
     assert not bit(rows, 0, 3)
@@ -63,7 +63,7 @@ def test_flights_extended_skylines_L99():
     assert rows[4].sum() == 0
 
 
-def test_flights_pairwise_masks_L77():
+def test_flights_pairwise_masks_L82():
     def mask(a, b, op):
         return "".join("1" if op(a[i], b[i]) else "0" for i in (2, 1, 0))
     f0, f1 = FLIGHTS[0], FLIGHTS[1]

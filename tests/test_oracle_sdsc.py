@@ -24,9 +24,9 @@ def test_flights_fig1a_and_line2():
     L, Lp = sdsc.sdsc(x)
     for delta_s, ids in GOLD["lattice"].items():
         assert L[int(delta_s)] == ids
-    # Alg. 2 line 2: L+[7] = S+_7 \ S_7 = {f4} (f4 is in S+ yet in no skyline, L99-101)
+    # Alg. 2 line 2: L+[7] = S+_7 \ S_7 = {f4} (f4 is in S+ yet in no skyline, L104-106)
     assert Lp[7] == [4]
-    # S+_3 = {f1, f2, f3, f4} (L99-101): L[3] U L+[3]
+    # S+_3 = {f1, f2, f3, f4} (L104-106): L[3] U L+[3]
     assert sorted(L[3] + Lp[3]) == GOLD["Splus3"]
     off, ids = sdsc.to_lattice(L, 3)
     assert off.tolist() == [0, 0, 1, 2, 5, 6, 9, 12, 16]
