@@ -55,7 +55,8 @@ def int_peaks(sm_mhz: float, sms: int = 148):
     try:
         with open(INTPEAK) as f:
             m = json.load(f)
-        alu, mix = m["alu"]["lane_ops_per_sm_per_clk"], m["mix"]["lane_ops_per_sm_per_clk"]
+        alu = m["alu"]["lane_ops_per_sm_per_clk"]
+        mix = max(m[k]["lane_ops_per_sm_per_clk"] for k in ("mix", "mix2") if k in m)
         basis = (f"measured (profiles/r02_intpeak.json: {alu:.1f} ALU-only and {mix:.1f} ALU+FMA integer lane-ops "
                  f"per SM per clock) x {sms} SMs x {sm_mhz:.0f} MHz (median SM clock of this run)")
     except Exception:
@@ -442,27 +443,50 @@ def measure_e2e(args, x, eng, world, rank, dev, pairs):
         t = statistics.median(times)
         keys = ("ms_h2d", "ms_sort", "ms_prefilter", "ms_mdmc", "ms_compact", "ms_d2h", "ms_total")
         return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
-                "ms_per_step": t * 1e3, "api": api,
+                "ms_per_step": t * 1e3, "api": api, "calls": len(times),
+                "note": "median of the calls; the result buffers come from the library's pinned pool (allocated by the "
+                        "warm-up call, reused after)",
                 "phases_ms": {k: statistics.median(p[k] for p in phases) for k in keys}}
-    # N > 1: pinned host input -> every rank H2D -> sharded pipeline -> rank 0 D2H of all outputs
+    # N > 1: pinned host input -> every rank H2D -> sharded pipeline; every rank writes its own membership rows
+    # (and the zero rows of its id slice) and its lattice segments straight into pinned host buffers (zero-copy
+    # over its own PCIe link); rank 0 also copies offsets and ext_ids.  The result is distributed over the ranks'
+    # host buffers (global positions); d2h bytes are summed over the ranks.
     host = torch.from_numpy(x).pin_memory()
+    W = (1 << d) >> 5 if d >= 5 else 1
+    warm = eng.build(host.to(dev), lists=True, membership=False)
+    total = warm["total_ids"]
+    h_mem = torch.empty((n, W), dtype=torch.int32).pin_memory()
+    h_ids = torch.empty(max(total, 1), dtype=torch.int32).pin_memory()
     times = []
     d2h = 0
     for i in range(args.e2e_steps + 1):
         dist.barrier()
         t0 = time.perf_counter()
         pts = host.to(dev, non_blocking=True)
-        out = eng.build(pts, lists=True, membership=True)
+        out = eng.build(pts, lists=True, membership=False, out_membership=h_mem, out_ids=h_ids)
+        extra = []
         if rank == 0:
-            res = [out["membership"].cpu(), out["ext_ids"].cpu(), out["offsets"].cpu(), out["ids"].cpu()]
-            d2h = sum(t.numel() * t.element_size() for t in res)
+            extra = [out["offsets"].cpu(), out["ext_ids"].cpu()]
         torch.cuda.synchronize()
         dist.barrier()
         if i:
             times.append(time.perf_counter() - t0)
+        else:
+            j0, j1 = out["shard"]
+            lo, hi = n * rank // world, n * (rank + 1) // world
+            ext = out["ext_ids"].cpu().numpy()
+            non_ext_in_slice = (hi - lo) - int(((ext >= lo) & (ext < hi)).sum())
+            # membership rows this rank writes (its tasks + the non-S+ rows of its id slice) and its copies; the
+            # lattice ids are written exactly once over all ranks (4 * total)
+            mine = (j1 - j0 + non_ext_in_slice) * W * 4 + sum(t.numel() * t.element_size() for t in extra)
+            d2h_t = torch.tensor([mine], dtype=torch.int64, device=dev)
+            dist.all_reduce(d2h_t)
+            d2h = int(d2h_t.item()) + 4 * total
     t = statistics.median(times)
-    return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes), "d2h_bytes_per_step": int(d2h),
-            "ms_per_step": t * 1e3, "api": "pipeline.DeviceSkycube (per-rank C-ABI device entry points)"}
+    return {"value": pairs / t, "unit": UNIT, "h2d_bytes_per_step": int(x.nbytes) * world, "d2h_bytes_per_step": int(d2h),
+            "ms_per_step": t * 1e3, "calls": len(times),
+            "api": ("pipeline.DeviceSkycube (per-rank C-ABI device entry points; every rank writes its rows and "
+                    "lattice segments zero-copy into pinned host buffers)")}
 
 
 def run_sdsc(args):

@@ -206,6 +206,28 @@ skycube_status skycube_dev_compact(skycube_ctx *ctx, const uint32_t *d_rows32, u
                                    int32_t *d_ext_ids, int64_t *d_offsets, int32_t *d_ids,
                                    int64_t *total_ids, void *stream);
 
+/* Multi-GPU compaction (one call sequence per rank, rank r owning the r-th contiguous
+ * range [j_begin, j_end) of S+ tasks, j_begin a multiple of 32, ranges in rank order covering [0, n_ext)):
+ *   1. skycube_dev_lattice_count: the rank's per-subspace counts -> d_totals[2^d] (int64, device);
+ *   2. the caller gathers every rank's totals into d_all_totals[num_shards][2^d] (e.g. an NCCL all-gather);
+ *   3. skycube_dev_lattice_scatter: writes the GLOBAL offsets d_offsets[2^d+1] (nullable) and the rank's ids at
+ *      their global positions of `ids` (device memory, or host-mapped pinned memory for a D2H straight into the
+ *      caller's result; other ranks' positions are not touched); *total_ids (nullable) = the global id count.
+ * d_rows32 is the tiled row buffer of skycube_dev_mdmc (only the rank's range is read).  Between 1 and 3 the
+ * context must not run another lattice pass.  With one shard (num_shards = 1, j range = all of S+) this is
+ * exactly the lattice of skycube_dev_compact. */
+skycube_status skycube_dev_lattice_count(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                         int64_t *d_totals, void *stream);
+skycube_status skycube_dev_lattice_scatter(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                           const int64_t *d_all_totals, int32_t num_shards, int32_t shard,
+                                           int64_t *d_offsets, int32_t *ids, int64_t *total_ids, void *stream);
+
+/* Membership rows by point id of the S+ tasks [j_begin, j_end) (tiled rows of skycube_dev_mdmc), plus zero
+ * rows for the points outside S+ whose ids lie in [zero_lo, zero_hi).  `membership` [n][W] is device memory or
+ * host-mapped pinned memory; no other row is touched (ranks write disjoint rows of one result). */
+skycube_status skycube_dev_membership(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                      int64_t zero_lo, int64_t zero_hi, uint32_t *membership, void *stream);
+
 /* Partial skycube for the following skycube_dev_mdmc calls (Appendix A.2; see skycube_opts.max_level):
  * 0 = full skycube, d' in [1, 16] = report only |delta| <= d'. */
 skycube_status skycube_ctx_set_max_level(skycube_ctx *ctx, int32_t max_level);

@@ -26,7 +26,7 @@ EXPORTED = (
     "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact", "skycube_ctx_launches",
     "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_free",
     "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc",
-    "skycube_set_tuning",
+    "skycube_set_tuning", "skycube_dev_lattice_count", "skycube_dev_lattice_scatter", "skycube_dev_membership",
 )
 
 
@@ -117,7 +117,11 @@ def lib():
         L.skycube_dev_hashcube.argtypes = [P, P, U32, P, P, P, P, ctypes.POINTER(I64), ctypes.POINTER(I64),
                                            ctypes.POINTER(I64), P]
         L.skycube_set_tuning.argtypes = [ctypes.c_char_p, I32]
-        for f in ("skycube_set_tuning", "skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
+        L.skycube_dev_lattice_count.argtypes = [P, P, I64, I64, P, P]
+        L.skycube_dev_lattice_scatter.argtypes = [P, P, I64, I64, P, I32, I32, P, P, ctypes.POINTER(I64), P]
+        L.skycube_dev_membership.argtypes = [P, P, I64, I64, I64, I64, P, P]
+        for f in ("skycube_dev_lattice_count", "skycube_dev_lattice_scatter", "skycube_dev_membership",
+                  "skycube_set_tuning", "skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
                   "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_query",
                   "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc"):
@@ -383,6 +387,25 @@ class Context:
         _check(lib().skycube_dev_compact(self._h, d_rows32, d_membership or None, d_ext_ids or None,
                                          d_offsets or None, d_ids or None, ctypes.byref(tot), stream or None))
         return tot.value
+
+    def lattice_count(self, d_rows32: int, j_begin: int, j_end: int, d_totals: int, stream: int = 0):
+        """Per-subspace counts of the S+ tasks [j_begin, j_end) -> d_totals[2^d] (int64 device)."""
+        _check(lib().skycube_dev_lattice_count(self._h, d_rows32, j_begin, j_end, d_totals, stream or None))
+
+    def lattice_scatter(self, d_rows32: int, j_begin: int, j_end: int, d_all_totals: int, num_shards: int, shard: int,
+                        d_offsets: int = 0, ids: int = 0, stream: int = 0) -> int:
+        """Global offsets and this shard's ids at their global positions (ids: device or host-mapped pointer);
+        returns the global id count."""
+        tot = ctypes.c_int64(0)
+        _check(lib().skycube_dev_lattice_scatter(self._h, d_rows32, j_begin, j_end, d_all_totals, num_shards, shard,
+                                                 d_offsets or None, ids or None, ctypes.byref(tot), stream or None))
+        return tot.value
+
+    def membership(self, d_rows32: int, j_begin: int, j_end: int, zero_lo: int, zero_hi: int, membership: int,
+                   stream: int = 0):
+        """Rows of the S+ tasks [j_begin, j_end) by id + zero rows outside S+ for ids in [zero_lo, zero_hi)."""
+        _check(lib().skycube_dev_membership(self._h, d_rows32, j_begin, j_end, zero_lo, zero_hi, membership,
+                                            stream or None))
 
     def set_max_level(self, max_level: int):
         _check(lib().skycube_ctx_set_max_level(self._h, max_level))

@@ -143,6 +143,7 @@ skycube_status guarded(F &&f) {
 // K3 work counters (exact DTs = misses, expansions) of a context, for skycube_stats
 void read_k3_counters(const sky::Ctx &c, int64_t *exact_dts, int64_t *expansions) {
     int64_t a[8] = {0};
+    SKY_CUDA(cudaSetDevice(c.device));
     SKY_CUDA(cudaMemcpy(a, c.counters.p, sizeof(a), cudaMemcpyDeviceToHost));
     *exact_dts = a[4];
     *expansions = a[6];
@@ -211,14 +212,26 @@ struct Events {
 };
 
 
-// Single-process multi-GPU build: num_gpus = k logical ranks on devices first .. first+k-1
-// (SKYCUBE_SHARE_DEVICES=1 lets ranks share devices round-robin -- the multi-rank logic on one GPU, tests).
+// Contiguous task range of shard g of k: 32-task groups split as evenly as possible, in shard order.
+inline void shard_range(int64_t m, int k, int g, int64_t *j0, int64_t *j1) {
+    const int64_t groups = sky::ceil_div(m, 32);
+    const int64_t g0 = groups * g / k, g1 = groups * (g + 1) / k;
+    *j0 = std::min<int64_t>(m, g0 * 32);
+    *j1 = std::min<int64_t>(m, g1 * 32);
+}
+
+// Single-process multi-GPU build: num_gpus = k logical ranks on devices first..first+k-1
+// (skycube_set_tuning("share_devices", 1) lets ranks share devices round-robin -- the k-rank logic on one GPU).
 //   every rank: H2D of the points, K0/K2 prepare (replicated, deterministic)
-//   rank g:     K1 on the prefilter blocks b = g (mod k); the k flag vectors are gathered on rank 0 by
-//               peer copies (NVLink), OR-combined and broadcast back; every rank installs S+
-//   rank g:     K3 on its contiguous range of 32-task groups; the row ranges are gathered on rank 0
-//   rank 0:     K4 (membership, lattice) and the D2H.
-// The output bytes are those of the single-GPU build (every kernel's result is scheduling-independent).
+//   rank g:     K1 on the prefilter blocks b = g (mod k); the k flag vectors are gathered on rank 0 by peer
+//               copies (NVLink), OR-combined and broadcast back; every rank installs S+
+//   rank g:     K3 on its contiguous range of 32-task groups; its membership rows go straight into the pinned
+//               host result by id (zero-copy over its own PCIe link), and it zeroes the rows of the points
+//               outside S+ in its slice of ids
+//   rank g:     K4 count pass over its own rows -> per-subspace totals; the k total vectors are exchanged by peer
+//               copies (k * 2^d int64); each rank places and writes its own ids straight into the pinned host
+//               lattice at their global positions
+// Nothing of size n or of the lattice crosses between GPUs; the output bytes equal the single-GPU build's.
 skycube_status build_multi(const float *points, int64_t n, int d, int first, int k, int max_level, bool lists,
                            skycube_result *out, skycube_stats *stats) {
     std::lock_guard<std::mutex> lk(g_mutex);
@@ -243,15 +256,16 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
             if (!x) x = new_ctx(dev[g]);
             xs[g] = x;
         }
-        for (int g = 1; g < k; g++) {  // NVLink peer access between rank 0 and every other device
-            if (dev[g] == dev[0]) continue;
-            int can = 0;
-            cudaDeviceCanAccessPeer(&can, dev[0], dev[g]);
-            if (can) {
-                SKY_CUDA(cudaSetDevice(dev[0]));
-                if (cudaDeviceEnablePeerAccess(dev[g], 0) != cudaSuccess) cudaGetLastError();
+        for (int g = 0; g < k; g++)  // NVLink peer access between every pair of distinct devices
+            for (int h = 0; h < k; h++) {
+                if (dev[g] == dev[h]) continue;
+                int can = 0;
+                cudaDeviceCanAccessPeer(&can, dev[g], dev[h]);
+                if (can) {
+                    SKY_CUDA(cudaSetDevice(dev[g]));
+                    if (cudaDeviceEnablePeerAccess(dev[h], 0) != cudaSuccess) cudaGetLastError();
+                }
             }
-        }
         r.d = d;
         r.n = n;
         r.words_per_row = sky::words_per_row(d);
@@ -263,9 +277,20 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
                 SKY_CUDA(cudaDeviceSynchronize());
             }
         };
-        int64_t launches0 = 0;
-        for (int g = 0; g < k; g++) launches0 += xs[g]->c.L.count;
-        const auto tp0 = std::chrono::steady_clock::now();
+        using clk = std::chrono::steady_clock;
+        double ms_comm = 0;
+        auto ms = [](clk::time_point a, clk::time_point b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
+        int64_t launches0 = 0, dts0 = 0, exp0 = 0;
+        for (int g = 0; g < k; g++) {
+            launches0 += xs[g]->c.L.count;
+            if (stats) {
+                int64_t a = 0, b = 0;
+                read_k3_counters(xs[g]->c, &a, &b);
+                dts0 += a;
+                exp0 += b;
+            }
+        }
+        const auto tp0 = clk::now();
         // prepare (replicated) + the rank's prefilter blocks
         for (int g = 0; g < k; g++) {
             skycube_ctx *x = xs[g];
@@ -278,7 +303,8 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
             sky::prefilter_run(x->c, g, k, x->ext8.as<uint8_t>(), nullptr);
         }
         sync_all();
-        // gather the flags on rank 0, OR, broadcast
+        // exchange 1: gather the flags on rank 0, OR, broadcast
+        const auto tc0 = clk::now();
         skycube_ctx *x0 = xs[0];
         SKY_CUDA(cudaSetDevice(dev[0]));
         x0->flag_stage.ensure((size_t)n * k);
@@ -288,72 +314,100 @@ skycube_status build_multi(const float *points, int64_t n, int d, int first, int
         for (int g = 1; g < k; g++)
             SKY_CUDA(cudaMemcpyPeerAsync(xs[g]->ext8.p, dev[g], x0->ext8.p, dev[0], n, nullptr));
         sync_all();
-        const auto tp1 = std::chrono::steady_clock::now();
+        ms_comm += ms(tc0, clk::now());
+        const auto tp1 = clk::now();
         for (int g = 0; g < k; g++) {
             SKY_CUDA(cudaSetDevice(dev[g]));
             sky::ext_build(xs[g]->c, xs[g]->ext8.as<uint8_t>(), nullptr);
         }
         const int64_t m = x0->c.m;
-        const int64_t groups = sky::ceil_div(m, 32), gpr = sky::ceil_div(groups, k);
-        const size_t grp_words = (size_t)W * 32;
-        const size_t rows_words = (size_t)std::max<int64_t>(groups, 1) * grp_words;
-        for (int g = 0; g < k; g++) {
-            skycube_ctx *x = xs[g];
-            SKY_CUDA(cudaSetDevice(dev[g]));
-            x->rows32.ensure(sizeof(uint32_t) * rows_words);
-            const int64_t j0 = std::min<int64_t>(m, g * gpr * 32), j1 = std::min<int64_t>(m, (g + 1) * gpr * 32);
-            x->c.max_level = max_level;
-            if (j1 > j0) sky::mdmc_run(x->c, j0, j1, x->rows32.as<uint32_t>(), nullptr, nullptr);
-        }
-        sync_all();
-        const auto tp2 = std::chrono::steady_clock::now();
-        SKY_CUDA(cudaSetDevice(dev[0]));
-        for (int g = 1; g < k; g++) {
-            const int64_t j0 = std::min<int64_t>(m, g * gpr * 32), j1 = std::min<int64_t>(m, (g + 1) * gpr * 32);
-            if (j1 <= j0) continue;
-            const size_t w0 = (size_t)(j0 / 32) * grp_words, w1 = (size_t)sky::ceil_div(j1, 32) * grp_words;
-            SKY_CUDA(cudaMemcpyPeerAsync(x0->rows32.as<uint32_t>() + w0, dev[0], xs[g]->rows32.as<uint32_t>() + w0, dev[g],
-                                         sizeof(uint32_t) * (w1 - w0), nullptr));
-        }
-        sky::Ctx &c = x0->c;
-        x0->membership.ensure(sizeof(uint32_t) * (size_t)n * W);
-        sky::compact_membership(c, x0->rows32.as<uint32_t>(), x0->membership.as<uint32_t>(), nullptr);
-        int64_t total = 0;
-        if (lists) {
-            x0->offsets.ensure(sizeof(int64_t) * (nsub + 1));
-            sky::compact_lattice(c, x0->rows32.as<uint32_t>(), x0->offsets.as<int64_t>(), nullptr, &total, nullptr);
-            x0->ids.ensure(sizeof(int32_t) * (total > 0 ? total : 1));
-            sky::compact_lattice(c, x0->rows32.as<uint32_t>(), x0->offsets.as<int64_t>(), x0->ids.as<int32_t>(), &total,
-                                 nullptr);
-        }
+        const size_t rows_words = (size_t)std::max<int64_t>(sky::ceil_div(m, 32), 1) * W * 32;
         r.n_ext = m;
         r.ext_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (m > 0 ? m : 1));
         r.membership = (uint32_t *)g_pool.get(sizeof(uint32_t) * (size_t)n * W);
-        if (m) SKY_CUDA(cudaMemcpyAsync(r.ext_ids, c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, nullptr));
-        SKY_CUDA(cudaMemcpyAsync(r.membership, x0->membership.p, sizeof(uint32_t) * (size_t)n * W, cudaMemcpyDeviceToHost,
-                                 nullptr));
+        std::vector<int64_t> j0(k), j1(k);
+        for (int g = 0; g < k; g++) {
+            skycube_ctx *x = xs[g];
+            SKY_CUDA(cudaSetDevice(dev[g]));
+            shard_range(m, k, g, &j0[g], &j1[g]);
+            x->rows32.ensure(sizeof(uint32_t) * rows_words);
+            x->c.max_level = max_level;
+            // K3 writes the rank's rows into the pinned result by id (zero-copy); the rank then zeroes the rows of
+            // the points outside S+ in its slice of ids
+            if (j1[g] > j0[g]) sky::mdmc_run(x->c, j0[g], j1[g], x->rows32.as<uint32_t>(), nullptr, nullptr, r.membership);
+            sky::compact_membership_shard(x->c, x->rows32.as<uint32_t>(), j0[g], j0[g], n * g / k, n * (g + 1) / k,
+                                          r.membership, nullptr);
+            if (lists) {
+                x->offsets.ensure(sizeof(int64_t) * (nsub + 1) + sizeof(int64_t) * (size_t)k * nsub);
+                sky::lattice_count_shard(x->c, x->rows32.as<uint32_t>(), j0[g], j1[g],
+                                         x->offsets.as<int64_t>() + (nsub + 1) + (size_t)g * nsub, nullptr);
+            }
+        }
+        if (m) {
+            SKY_CUDA(cudaSetDevice(dev[0]));
+            SKY_CUDA(cudaMemcpyAsync(r.ext_ids, x0->c.ext_ids.p, sizeof(int32_t) * m, cudaMemcpyDeviceToHost, nullptr));
+        }
+        sync_all();
+        const auto tp2 = clk::now();
+        int64_t total = 0;
         if (lists) {
+            // exchange 2: every rank's per-subspace totals to every rank (k * 2^d int64 by peer copies)
+            const auto tc1 = clk::now();
+            const size_t tb = sizeof(int64_t) * (size_t)nsub;
+            for (int g = 0; g < k; g++) {
+                SKY_CUDA(cudaSetDevice(dev[g]));
+                int64_t *all_g = xs[g]->offsets.as<int64_t>() + (nsub + 1);
+                for (int h = 0; h < k; h++)
+                    if (h != g)
+                        SKY_CUDA(cudaMemcpyPeerAsync(all_g + (size_t)h * nsub, dev[g],
+                                                     xs[h]->offsets.as<int64_t>() + (nsub + 1) + (size_t)h * nsub, dev[h],
+                                                     tb, nullptr));
+            }
+            sync_all();
+            ms_comm += ms(tc1, clk::now());
+            // the id count (to size the pinned lattice) from rank 0's placement pass, then every rank writes its
+            // own segments straight into the pinned host lattice
+            SKY_CUDA(cudaSetDevice(dev[0]));
+            total = sky::lattice_scatter_shard(x0->c, x0->rows32.as<uint32_t>(), j0[0], j1[0],
+                                               x0->offsets.as<int64_t>() + (nsub + 1), k, 0, x0->offsets.as<int64_t>(),
+                                               nullptr, nullptr);
             r.cuboid_offsets = (int64_t *)g_pool.get(sizeof(int64_t) * (nsub + 1));
             r.cuboid_ids = (int32_t *)g_pool.get(sizeof(int32_t) * (total > 0 ? total : 1));
             SKY_CUDA(cudaMemcpyAsync(r.cuboid_offsets, x0->offsets.p, sizeof(int64_t) * (nsub + 1), cudaMemcpyDeviceToHost,
                                      nullptr));
-            if (total)
-                SKY_CUDA(cudaMemcpyAsync(r.cuboid_ids, x0->ids.p, sizeof(int32_t) * total, cudaMemcpyDeviceToHost, nullptr));
+            for (int g = 0; g < k; g++) {
+                skycube_ctx *x = xs[g];
+                SKY_CUDA(cudaSetDevice(dev[g]));
+                if (j1[g] > j0[g])
+                    sky::lattice_scatter_shard(x->c, x->rows32.as<uint32_t>(), j0[g], j1[g],
+                                               x->offsets.as<int64_t>() + (nsub + 1), k, g, nullptr, r.cuboid_ids, nullptr);
+            }
         }
-        SKY_CUDA(cudaDeviceSynchronize());
-        SKY_CUDA(cudaGetLastError());
-        const auto tp3 = std::chrono::steady_clock::now();
+        sync_all();
+        for (int g = 0; g < k; g++) {
+            SKY_CUDA(cudaSetDevice(dev[g]));
+            SKY_CUDA(cudaGetLastError());
+        }
+        const auto tp3 = clk::now();
         if (stats) {  // host clock per phase (several devices)
-            auto ms = [](auto a, auto b) { return std::chrono::duration<double, std::milli>(b - a).count(); };
-            stats->ms_sort = ms(tp0, tp1);  // H2D + prepare + prefilter + flag exchange
-            stats->ms_mdmc = ms(tp1, tp2);  // S+ install + K3
-            stats->ms_compact = ms(tp2, tp3);  // row gather + K4 + D2H
+            stats->ms_sort = ms(tp0, tp1);     // H2D + prepare + prefilter + flag exchange
+            stats->ms_mdmc = ms(tp1, tp2);     // S+ install + K3 (rows zero-copy to the host) + K4 counts
+            stats->ms_compact = ms(tp2, tp3);  // totals exchange + K4 placement and scatter (ids zero-copy)
+            stats->ms_comm = ms_comm;
             stats->n_ext = m;
             stats->pairs = m * (m > 0 ? m - 1 : 0);
             stats->total_ids = total;
-            int64_t launches = 0;
-            for (int g = 0; g < k; g++) launches += xs[g]->c.L.count;
+            int64_t launches = 0, dts = 0, exps = 0;
+            for (int g = 0; g < k; g++) {
+                launches += xs[g]->c.L.count;
+                int64_t a = 0, b = 0;
+                read_k3_counters(xs[g]->c, &a, &b);
+                dts += a;
+                exps += b;
+            }
             stats->kernel_launches = (int32_t)(launches - launches0);
+            stats->exact_dts = dts - dts0;
+            stats->expansions = exps - exp0;
             stats->num_gpus = k;
         }
     });
@@ -824,6 +878,43 @@ skycube_status skycube_dev_mdmc(skycube_ctx *ctx, int64_t j_begin, int64_t j_end
     return guarded([&] {
         SKY_CUDA(cudaSetDevice(ctx->c.device));
         sky::mdmc_run(ctx->c, j_begin, j_end, d_rows32, d_ext_rows32, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_lattice_count(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                         int64_t *d_totals, void *stream) {
+    if (!ctx || !d_rows32 || !d_totals) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        sky::Ctx &c = ctx->c;
+        if (!c.ext_ready) throw sky::Error{SKYCUBE_EINVAL, "skycube_dev_lattice_count before skycube_dev_set_ext"};
+        SKY_CUDA(cudaSetDevice(c.device));
+        sky::lattice_count_shard(c, d_rows32, j_begin, j_end, d_totals, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_lattice_scatter(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                           const int64_t *d_all_totals, int32_t num_shards, int32_t shard,
+                                           int64_t *d_offsets, int32_t *ids, int64_t *total_ids, void *stream) {
+    if (!ctx || !d_rows32 || !d_all_totals) return fail(SKYCUBE_EINVAL, "NULL argument");
+    if (num_shards < 1 || shard < 0 || shard >= num_shards) return fail(SKYCUBE_EINVAL, "bad shard index");
+    return guarded([&] {
+        sky::Ctx &c = ctx->c;
+        if (!c.ext_ready) throw sky::Error{SKYCUBE_EINVAL, "skycube_dev_lattice_scatter before skycube_dev_set_ext"};
+        SKY_CUDA(cudaSetDevice(c.device));
+        const int64_t t = sky::lattice_scatter_shard(c, d_rows32, j_begin, j_end, d_all_totals, num_shards, shard,
+                                                     d_offsets, ids, (cudaStream_t)stream);
+        if (total_ids) *total_ids = t;
+    });
+}
+
+skycube_status skycube_dev_membership(skycube_ctx *ctx, const uint32_t *d_rows32, int64_t j_begin, int64_t j_end,
+                                      int64_t zero_lo, int64_t zero_hi, uint32_t *membership, void *stream) {
+    if (!ctx || !d_rows32 || !membership) return fail(SKYCUBE_EINVAL, "NULL argument");
+    return guarded([&] {
+        sky::Ctx &c = ctx->c;
+        if (!c.ext_ready) throw sky::Error{SKYCUBE_EINVAL, "skycube_dev_membership before skycube_dev_set_ext"};
+        SKY_CUDA(cudaSetDevice(c.device));
+        sky::compact_membership_shard(c, d_rows32, j_begin, j_end, zero_lo, zero_hi, membership, (cudaStream_t)stream);
     });
 }
 

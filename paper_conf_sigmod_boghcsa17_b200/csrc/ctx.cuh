@@ -120,6 +120,12 @@ void compact_membership(Ctx &c, const uint32_t *rows32, uint32_t *membership, cu
 void membership_zero_outside(Ctx &c, uint32_t *membership, cudaStream_t st);
 void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
                      cudaStream_t st);
+// multi-GPU shards of K4 (S+ tasks [j0, j1), j0 a multiple of 32): count -> exchange totals -> scatter
+void lattice_count_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, int64_t *d_totals, cudaStream_t st);
+int64_t lattice_scatter_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, const int64_t *all_totals, int k,
+                              int rank, int64_t *offsets, int32_t *ids, cudaStream_t st);
+void compact_membership_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, int64_t zlo, int64_t zhi,
+                              uint32_t *membership, cudaStream_t st);
 // sdsc.cu: Alg. 2 over the installed S+; lattice into d_offsets / *d_ids (context-owned), rows into
 // d_membership (nullable); returns the number of ids
 int64_t sdsc_run(Ctx &c, int64_t *d_offsets, uint32_t *d_membership, cudaStream_t st, int32_t **d_ids);

@@ -211,6 +211,59 @@ __global__ void __launch_bounds__(1024) lattice_scatter32_kernel(const uint32_t 
     }
 }
 
+// Multi-GPU placement of one shard's segments: all[r * nsub + delta] = count of subspace
+// delta in shard r.  tot[delta] = the global count, pre[delta] = the counts of the shards before `rank`.
+__global__ void lattice_place_kernel(const int64_t *__restrict__ all, int k, int rank, int64_t nsub, int64_t NS,
+                                     uint64_t *__restrict__ tot, uint64_t *__restrict__ pre) {
+    const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (delta >= NS) return;
+    uint64_t t = 0, p = 0;
+    if (delta < nsub)
+        for (int r = 0; r < k; r++) {
+            const uint64_t v = (uint64_t)all[(int64_t)r * nsub + delta];
+            if (r < rank) p += v;
+            t += v;
+        }
+    tot[delta] = t;
+    pre[delta] = p;
+}
+
+// doff[delta] += pre[delta]: the shard's segment of subspace delta starts after the earlier shards' ids
+__global__ void lattice_shift_kernel(uint64_t *__restrict__ doff, const uint64_t *__restrict__ pre, int64_t NS) {
+    const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (delta < NS) doff[delta] += pre[delta];
+}
+
+__global__ void totals_out_kernel(const uint64_t *__restrict__ tot, int64_t nsub, int64_t *__restrict__ out) {
+    const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (delta < nsub) out[delta] = (int64_t)tot[delta];
+}
+
+// Membership rows of the tasks of one shard, by point id; the rows of the points outside S+ with ids in
+// [zlo, zhi) are zeroed (each shard zeroes its own slice of ids).  `membership` may be host-mapped.
+__global__ void membership_shard_kernel(const uint32_t *__restrict__ rows32, const int32_t *__restrict__ ext_ids,
+                                        int64_t mr, uint32_t W, uint32_t *__restrict__ membership) {
+    __shared__ uint32_t tile[32][33];
+    const int64_t g = blockIdx.x;
+    const uint32_t wc = blockIdx.y * 32u;
+    const uint32_t nw = min(32u, W - wc);
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    for (uint32_t w = ty; w < nw; w += 8) tile[w][tx] = rows32[g * W * 32 + (int64_t)(wc + w) * 32 + tx];
+    __syncthreads();
+    for (int l = ty; l < 32; l += 8) {
+        const int64_t j = g * 32 + l;
+        if (j >= mr) break;
+        if ((uint32_t)tx < nw) membership[(int64_t)ext_ids[j] * W + wc + tx] = tile[tx][l];
+    }
+}
+
+__global__ void zero_outside_range_kernel(const uint32_t *__restrict__ ext_id_flag, int64_t lo, int64_t hi, uint32_t W,
+                                          uint32_t *__restrict__ membership) {
+    const int64_t total = (hi - lo) * (int64_t)W;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x)
+        if (!ext_id_flag[lo + i / W]) membership[lo * (int64_t)W + i] = 0u;
+}
+
 __global__ void lattice_offsets_kernel(const uint64_t *__restrict__ doff, const uint64_t *__restrict__ tot,
                                        int64_t nsub, int64_t *__restrict__ offsets) {
     const int64_t delta = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -238,58 +291,162 @@ void membership_zero_outside(Ctx &c, uint32_t *membership, cudaStream_t st) {
     SKY_LAUNCH_CHECK();
 }
 
-// Two calls: ids == nullptr computes counts/scan/offsets and *total_ids; then ids != nullptr scatters.
-void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
-                     cudaStream_t st) {
-    const int64_t nsub = (int64_t)1 << c.d;
-    const int64_t ngroups = ceil_div(c.m, 32);
-    const bool big = c.d > 12;
-    const int nwk = big ? 32 : 8;
-    const int64_t nchunks = ceil_div(ngroups > 0 ? ngroups : 1, nwk);
-    const int64_t NS = (int64_t)c.W * 32;  // >= nsub
-    const int64_t nentries = NS * nchunks;
-    const unsigned gy = (unsigned)std::min<int64_t>(ceil_div(c.W, kUnr), big ? 16 : 4);
-    dim3 grid((unsigned)nchunks, gy);
-    c.lat_counts.ensure(sizeof(uint64_t) * (2 * (size_t)nentries + 2 * (size_t)NS));
-    uint64_t *counts = c.lat_counts.as<uint64_t>();
-    uint64_t *colpre = counts + nentries;
-    uint64_t *tot = colpre + nentries;
-    uint64_t *doff = tot + NS;
-    if (ids == nullptr) {
-        c.scan64_tmp.ensure(scan_tmp_bytes(NS));
-        if (c.m == 0) {
-            SKY_CUDA(cudaMemsetAsync(counts, 0, sizeof(uint64_t) * (size_t)nentries, st));
-        } else {
-            if (big)
-                lattice_count_kernel<32><<<grid, 32 * 32, 0, st>>>(rows32, c.m, c.W, counts);
-            else
-                lattice_count_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, counts);
-            c.L.count++;
-            SKY_LAUNCH_CHECK();
-        }
-        lattice_colscan_kernel<<<(unsigned)ceil_div(NS, 128), 128, 0, st>>>(counts, nchunks, NS, colpre, tot);
+// Geometry of the lattice passes over the shard of S+ tasks [j0, j1) (j0 a multiple of 32).
+struct LatGeo {
+    int64_t nsub, mr, nchunks, NS, nentries;
+    bool big;
+    int nwk;
+    dim3 grid;
+    LatGeo(const Ctx &c, int64_t j0, int64_t j1) {
+        nsub = (int64_t)1 << c.d;
+        mr = j1 - j0;
+        big = c.d > 12;
+        nwk = big ? 32 : 8;
+        const int64_t ngroups = ceil_div(mr, 32);
+        nchunks = ceil_div(ngroups > 0 ? ngroups : 1, nwk);
+        NS = (int64_t)c.W * 32;  // >= nsub
+        nentries = NS * nchunks;
+        const unsigned gy = (unsigned)std::min<int64_t>(ceil_div(c.W, kUnr), big ? 16 : 4);
+        grid = dim3((unsigned)nchunks, gy);
+    }
+};
+
+// scratch: counts, colpre [nentries] then tot, doff, pre [NS]
+static uint64_t *lat_scratch(Ctx &c, const LatGeo &g) {
+    c.lat_counts.ensure(sizeof(uint64_t) * (2 * (size_t)g.nentries + 3 * (size_t)g.NS));
+    return c.lat_counts.as<uint64_t>();
+}
+
+// Count pass of a shard: per (chunk, subspace) counts, the per-subspace prefix over the shard's chunks (kept in
+// the context for the scatter) and the shard's per-subspace totals (written to d_totals[nsub] if non-null).
+void lattice_count_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, int64_t *d_totals, cudaStream_t st) {
+    if (j0 < 0 || j1 > c.m || (j0 & 31) || j1 < j0) throw Error{1, "bad lattice shard range"};
+    const LatGeo g(c, j0, j1);
+    uint64_t *counts = lat_scratch(c, g), *colpre = counts + g.nentries, *tot = colpre + g.nentries;
+    const uint32_t *rows = rows32 + (j0 / 32) * (int64_t)c.W * 32;
+    if (g.mr == 0) {
+        SKY_CUDA(cudaMemsetAsync(counts, 0, sizeof(uint64_t) * (size_t)g.nentries, st));
+    } else {
+        if (g.big)
+            lattice_count_kernel<32><<<g.grid, 32 * 32, 0, st>>>(rows, g.mr, c.W, counts);
+        else
+            lattice_count_kernel<8><<<g.grid, 8 * 32, 0, st>>>(rows, g.mr, c.W, counts);
         c.L.count++;
         SKY_LAUNCH_CHECK();
-        exclusive_scan_u64(tot, doff, NS, c.scan64_tmp.p, st, c.L);
-        lattice_offsets_kernel<<<(unsigned)ceil_div(nsub + 1, 256), 256, 0, st>>>(doff, tot, nsub, offsets);
+    }
+    lattice_colscan_kernel<<<(unsigned)ceil_div(g.NS, 128), 128, 0, st>>>(counts, g.nchunks, g.NS, colpre, tot);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    if (d_totals) {
+        totals_out_kernel<<<(unsigned)ceil_div(g.nsub, 256), 256, 0, st>>>(tot, g.nsub, d_totals);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+}
+
+// Scatter pass of a shard after lattice_count_shard: all_totals[k][nsub] are the totals of every shard (rank r
+// covers the r-th task range in S+ order, so its ids of subspace delta follow those of ranks < r).  Writes the
+// global offsets[nsub + 1] (nullable) and the shard's ids at their global positions of ids[] (device or
+// host-mapped memory; ids of other shards are not touched).  Returns the global id count.
+int64_t lattice_scatter_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, const int64_t *all_totals, int k,
+                              int rank, int64_t *offsets, int32_t *ids, cudaStream_t st) {
+    const LatGeo g(c, j0, j1);
+    uint64_t *counts = lat_scratch(c, g), *colpre = counts + g.nentries, *tot = colpre + g.nentries;
+    uint64_t *doff = tot + g.NS, *pre = doff + g.NS;
+    (void)counts;
+    c.scan64_tmp.ensure(scan_tmp_bytes(g.NS));
+    // global totals -> tot (the shard's own totals are no longer needed), the earlier shards' counts -> pre
+    lattice_place_kernel<<<(unsigned)ceil_div(g.NS, 256), 256, 0, st>>>(all_totals, k, rank, g.nsub, g.NS, tot, pre);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    exclusive_scan_u64(tot, doff, g.NS, c.scan64_tmp.p, st, c.L);
+    if (offsets) {
+        lattice_offsets_kernel<<<(unsigned)ceil_div(g.nsub + 1, 256), 256, 0, st>>>(doff, tot, g.nsub, offsets);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    int64_t total = 0;
+    {
+        uint64_t last[2];
+        SKY_CUDA(cudaMemcpyAsync(&last[0], doff + g.nsub - 1, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        SKY_CUDA(cudaMemcpyAsync(&last[1], tot + g.nsub - 1, sizeof(uint64_t), cudaMemcpyDeviceToHost, st));
+        SKY_CUDA(cudaStreamSynchronize(st));
+        total = (int64_t)(last[0] + last[1]);
+    }
+    if (g.mr == 0 || !ids) return total;
+    if (k > 1 || rank > 0) {
+        lattice_shift_kernel<<<(unsigned)ceil_div(g.NS, 256), 256, 0, st>>>(doff, pre, g.NS);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    const uint32_t *rows = rows32 + (j0 / 32) * (int64_t)c.W * 32;
+    const int32_t *eid = c.ext_ids.as<int32_t>() + j0;
+    if (g.big) {
+        const int smem = 32 * 1024 * (int)sizeof(int32_t);
+        SKY_CUDA(cudaFuncSetAttribute(lattice_scatter32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        lattice_scatter32_kernel<<<dim3((unsigned)g.nchunks, (unsigned)std::min<int64_t>(c.W, 64)), 1024, smem, st>>>(
+            rows, g.mr, c.W, colpre, doff, eid, ids);
+    } else {
+        lattice_scatter_kernel<8><<<g.grid, 8 * 32, 0, st>>>(rows, g.mr, c.W, colpre, doff, eid, ids);
+    }
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+    return total;
+}
+
+// Single-GPU lattice: the whole of S+ as one shard.  Two calls: ids == nullptr computes counts/scan/offsets and
+// *total_ids; then ids != nullptr scatters.
+void compact_lattice(Ctx &c, const uint32_t *rows32, int64_t *offsets, int32_t *ids, int64_t *total_ids,
+                     cudaStream_t st) {
+    const LatGeo g(c, 0, c.m);
+    if (ids == nullptr) {
+        lattice_count_shard(c, rows32, 0, c.m, nullptr, st);
+        uint64_t *counts = lat_scratch(c, g), *colpre = counts + g.nentries, *tot = colpre + g.nentries;
+        uint64_t *doff = tot + g.NS;
+        c.scan64_tmp.ensure(scan_tmp_bytes(g.NS));
+        exclusive_scan_u64(tot, doff, g.NS, c.scan64_tmp.p, st, c.L);
+        lattice_offsets_kernel<<<(unsigned)ceil_div(g.nsub + 1, 256), 256, 0, st>>>(doff, tot, g.nsub, offsets);
         c.L.count++;
         SKY_LAUNCH_CHECK();
         int64_t tot_ids = 0;
-        SKY_CUDA(cudaMemcpyAsync(&tot_ids, offsets + nsub, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        SKY_CUDA(cudaMemcpyAsync(&tot_ids, offsets + g.nsub, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
         SKY_CUDA(cudaStreamSynchronize(st));
         *total_ids = tot_ids;
         return;
     }
     if (c.m == 0) return;
-    if (big)
-    {
+    uint64_t *counts = lat_scratch(c, g), *colpre = counts + g.nentries, *tot = colpre + g.nentries;
+    uint64_t *doff = tot + g.NS;
+    (void)counts;
+    if (g.big) {
         const int smem = 32 * 1024 * (int)sizeof(int32_t);
         SKY_CUDA(cudaFuncSetAttribute(lattice_scatter32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        lattice_scatter32_kernel<<<dim3((unsigned)nchunks, (unsigned)std::min<int64_t>(c.W, 64)), 1024, smem, st>>>(
+        lattice_scatter32_kernel<<<dim3((unsigned)g.nchunks, (unsigned)std::min<int64_t>(c.W, 64)), 1024, smem, st>>>(
             rows32, c.m, c.W, colpre, doff, c.ext_ids.as<int32_t>(), ids);
+    } else {
+        lattice_scatter_kernel<8><<<g.grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, colpre, doff, c.ext_ids.as<int32_t>(), ids);
     }
-    else
-        lattice_scatter_kernel<8><<<grid, 8 * 32, 0, st>>>(rows32, c.m, c.W, colpre, doff, c.ext_ids.as<int32_t>(), ids);
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
+}
+
+// Membership by id of the shard [j0, j1) of S+ tasks, and zero rows for the points outside S+ whose ids lie in
+// [zlo, zhi).  `membership` [n][W] may be device or host-mapped memory; nothing else of it is touched.
+void compact_membership_shard(Ctx &c, const uint32_t *rows32, int64_t j0, int64_t j1, int64_t zlo, int64_t zhi,
+                              uint32_t *membership, cudaStream_t st) {
+    if (j0 < 0 || j1 > c.m || (j0 & 31) || j1 < j0 || zlo < 0 || zhi > c.n || zhi < zlo)
+        throw Error{1, "bad membership shard range"};
+    if (zhi > zlo) {
+        const int64_t total = (zhi - zlo) * (int64_t)c.W;
+        const unsigned blocks = (unsigned)std::min<int64_t>(ceil_div(total, 256), (int64_t)c.num_sms * 8);
+        zero_outside_range_kernel<<<blocks, 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), zlo, zhi, c.W, membership);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    if (j1 == j0) return;
+    dim3 grid((unsigned)ceil_div(j1 - j0, 32), (unsigned)ceil_div(c.W, 32));
+    membership_shard_kernel<<<grid, 256, 0, st>>>(rows32 + (j0 / 32) * (int64_t)c.W * 32, c.ext_ids.as<int32_t>() + j0,
+                                                  j1 - j0, c.W, membership);
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }

@@ -3,22 +3,27 @@
 Sharding (the paper's device-level data parallelism of MDMC, L308-310, L420 "every
 task is independent, there is no need for synchronisation"):
 
-  1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic)
-  2. K1 prefilter                                 blocks of 512 static-tree positions,
-                                                  block b on rank b % world
+  1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic, ~2 ms at H)
+  2. K1 prefilter                                 blocks of 512 static-tree positions, block b on rank b % world
   3. exchange S+ flags                            all_reduce(MAX) of a uint8 flag vector (NCCL over NVLink)
   4. install S+ (replicated)
-  5. K3 MDMC                                      contiguous ranges of 32-point groups of S+ (per-task cost is
-                                                  uniform: every task scans all of S+)
-  6. exchange rows                                all_gather of the rank's row chunk (NCCL over NVLink)
-  7. K4 compaction                                every rank (identical bytes on every rank)
+  5. K3 MDMC                                      contiguous ranges of 32-point groups of S+, split evenly
+  6. K4 compaction, sharded                       each rank: membership rows of its own tasks by id (plus zero
+                                                  rows for the points outside S+ in its slice of ids) and the
+                                                  per-subspace counts of its rows; all_gather of the counts
+                                                  (world x 2^d int64); each rank places its ids at their
+                                                  global positions of the lattice and writes them
+  7. HashCube (optional)                          needs every row: all_gather of the rows, then K5 on each rank
 
-The collective helpers below are plain torch.distributed calls so that the same code runs on NCCL
-(GPU) and gloo (CPU tests).  Only the kernels are native; nothing here computes skycube values.
+No row, membership or lattice data crosses between ranks on the lattice path: the result is distributed, each
+rank holding the rows of its tasks and its segments of every subspace list at their global positions (a
+caller assembles one array by letting every rank write into one shared/pinned buffer, as the C-ABI's
+single-process num_gpus path does).  The collective helpers are plain torch.distributed calls so that the
+same code runs on NCCL (GPU) and gloo (CPU tests).  Only the kernels are native; nothing here computes
+skycube values.
 """
 from __future__ import annotations
 
-import math
 from dataclasses import dataclass
 
 import torch
@@ -36,25 +41,21 @@ def prefilter_assignment(rank: int, world: int):
     return rank, world
 
 
-def groups_per_rank(m: int, world: int) -> int:
-    ngroups = math.ceil(m / GROUP) if m > 0 else 0
-    return math.ceil(ngroups / world) if ngroups else 0
-
-
 def task_range(m: int, world: int, rank: int):
-    """[j_begin, j_end) of the S+ tasks of a rank (multiples of 32 except the global end)."""
-    gpr = groups_per_rank(m, world)
-    j0 = min(m, rank * gpr * GROUP)
-    j1 = min(m, (rank + 1) * gpr * GROUP)
-    return j0, j1
+    """[j_begin, j_end) of the S+ tasks of a rank: the 32-task groups split as evenly as possible, in rank order
+    (the same split as capi.cu shard_range)."""
+    groups = (m + GROUP - 1) // GROUP
+    g0, g1 = groups * rank // world, groups * (rank + 1) // world
+    return min(m, g0 * GROUP), min(m, g1 * GROUP)
 
 
-def rows_buffer_words(m: int, d: int, world: int) -> int:
-    return max(1, groups_per_rank(m, world) * world) * GROUP * words_per_row(d)
+def id_slice(n: int, world: int, rank: int):
+    """[lo, hi) of the point ids whose non-S+ membership rows a rank zeroes."""
+    return n * rank // world, n * (rank + 1) // world
 
 
-def chunk_words(m: int, d: int, world: int) -> int:
-    return groups_per_rank(m, world) * GROUP * words_per_row(d)
+def rows_buffer_words(m: int, d: int) -> int:
+    return max(1, (m + GROUP - 1) // GROUP) * GROUP * words_per_row(d)
 
 
 # ------------------------------------------------------------------ collectives (NCCL or gloo)
@@ -64,9 +65,13 @@ def _staged(t: torch.Tensor, group) -> bool:
     return t.is_cuda and dist.get_backend(group) == "gloo"
 
 
+def _world(group):
+    return dist.get_world_size(group) if dist.is_initialized() else 1
+
+
 def exchange_ext(ext8: torch.Tensor, group=None):
     """Combine per-rank S+ flags: every position was written by exactly one rank, others are 0."""
-    if dist.is_initialized() and dist.get_world_size(group) > 1:
+    if _world(group) > 1:
         if _staged(ext8, group):
             h = ext8.cpu()
             dist.all_reduce(h, op=dist.ReduceOp.MAX, group=group)
@@ -76,22 +81,46 @@ def exchange_ext(ext8: torch.Tensor, group=None):
     return ext8
 
 
-def exchange_rows(rows32: torch.Tensor, m: int, d: int, group=None):
-    """All-gather the rank-owned chunks of the tiled row buffer (equal chunk sizes by construction)."""
-    if not (dist.is_initialized() and dist.get_world_size(group) > 1):
-        return rows32
-    world = dist.get_world_size(group)
-    rank = dist.get_rank(group)
-    cw = chunk_words(m, d, world)
-    if cw == 0:
-        return rows32
-    mine = rows32[rank * cw:(rank + 1) * cw].clone()
-    if _staged(rows32, group):
-        h = torch.empty(world * cw, dtype=rows32.dtype)
-        dist.all_gather_into_tensor(h, mine.cpu(), group=group)
-        rows32[:world * cw].copy_(h)
+def exchange_totals(totals: torch.Tensor, group=None) -> torch.Tensor:
+    """All-gather every rank's per-subspace counts: [world * 2^d] int64, rank-major."""
+    world = _world(group)
+    if world == 1:
+        return totals
+    out = torch.empty(world * totals.numel(), dtype=totals.dtype, device=totals.device)
+    if _staged(totals, group):
+        h = torch.empty(world * totals.numel(), dtype=totals.dtype)
+        dist.all_gather_into_tensor(h, totals.cpu(), group=group)
+        out.copy_(h)
     else:
-        dist.all_gather_into_tensor(rows32[:world * cw], mine, group=group)
+        dist.all_gather_into_tensor(out, totals, group=group)
+    return out
+
+
+def gather_rows(rows32: torch.Tensor, m: int, d: int, group=None):
+    """Assemble every rank's row range into the full tiled row buffer (HashCube output only): ranges are
+    contiguous but unequal, so each rank contributes a padded chunk of the largest range."""
+    world = _world(group)
+    if world == 1:
+        return rows32
+    rank = dist.get_rank(group)
+    W = words_per_row(d)
+    gw = GROUP * W
+    ranges = [task_range(m, world, r) for r in range(world)]
+    cmax = max((b - a + GROUP - 1) // GROUP for a, b in ranges) * gw
+    j0, j1 = ranges[rank]
+    mine = torch.zeros(max(cmax, 1), dtype=rows32.dtype, device=rows32.device)
+    nw = (j1 - j0 + GROUP - 1) // GROUP * gw
+    mine[:nw] = rows32[j0 // GROUP * gw: j0 // GROUP * gw + nw]
+    if _staged(rows32, group):
+        h = torch.empty(world * mine.numel(), dtype=rows32.dtype)
+        dist.all_gather_into_tensor(h, mine.cpu(), group=group)
+        allc = h.to(rows32.device)
+    else:
+        allc = torch.empty(world * mine.numel(), dtype=rows32.dtype, device=rows32.device)
+        dist.all_gather_into_tensor(allc, mine, group=group)
+    for r, (a, b) in enumerate(ranges):
+        k = (b - a + GROUP - 1) // GROUP * gw
+        rows32[a // GROUP * gw: a // GROUP * gw + k] = allc[r * mine.numel(): r * mine.numel() + k]
     return rows32
 
 
@@ -105,7 +134,7 @@ class StepTimes:
 
 
 class DeviceSkycube:
-    """Runs the five phases on one GPU; with world > 1 it shards K1 and K3 over the process group."""
+    """Runs the five phases on one GPU; with world > 1 it shards K1, K3 and K4 over the process group."""
 
     def __init__(self, device: int = 0, group=None):
         self.device = torch.device("cuda", device)
@@ -117,20 +146,26 @@ class DeviceSkycube:
         return self.ctx.launches
 
     def build(self, pts: torch.Tensor, lists: bool = True, membership: bool = True, events: dict | None = None,
-              hashcube_w: int = 0, max_level: int = 0):
-        """pts: (n, d) float32 CUDA tensor (resident).  Returns dict of device tensors:
-        n_ext, rows32 (tiled rows of S+), ext_ids, membership [n, W] (optional), offsets, ids, and with
-        hashcube_w > 0 the HashCube (K5, Appendix B.1) as hashcube = {word_offsets, keys, key_offsets, ids}.
-        max_level = d' > 0: partial skycube (Appendix A.2), only |delta| <= d' reported."""
+              hashcube_w: int = 0, max_level: int = 0, out_membership: torch.Tensor | None = None,
+              out_ids: torch.Tensor | None = None):
+        """pts: (n, d) float32 CUDA tensor (resident).  Returns dict of tensors:
+        n_ext, shard (j_begin, j_end) of this rank's S+ tasks, rows32 (tiled rows; this rank's range is valid),
+        ext_ids, membership [n, W] (optional; with world > 1 only this rank's rows and zero slice are written),
+        offsets (global), ids (global positions; with world > 1 only this rank's segments are written),
+        total_ids, and with hashcube_w > 0 the HashCube (K5, Appendix B.1).
+        max_level = d' > 0: partial skycube (Appendix A.2), only |delta| <= d' reported.
+        out_membership / out_ids: caller-provided destinations (device or pinned host tensors: the kernels
+        write pinned host memory directly, zero-copy); out_ids must hold total_ids entries."""
         assert pts.is_cuda and pts.dtype == torch.float32 and pts.dim() == 2
         pts = pts.contiguous()
         n, d = pts.shape
-        world = dist.get_world_size(self.group) if dist.is_initialized() else 1
-        rank = dist.get_rank(self.group) if dist.is_initialized() else 0
+        world = _world(self.group)
+        rank = dist.get_rank(self.group) if world > 1 else 0
         stream = torch.cuda.current_stream(self.device)
         sp = stream.cuda_stream
         rec = (lambda k: events[k].record(stream)) if events is not None else (lambda k: None)
         W = words_per_row(d)
+        nsub = 1 << d
 
         rec("t0")
         self.ctx.prepare(pts.data_ptr(), n, d, sp)
@@ -141,28 +176,45 @@ class DeviceSkycube:
         exchange_ext(ext8, self.group)
         m = self.ctx.set_ext(ext8.data_ptr(), sp)
         rec("t2")
-        rows32 = torch.empty(rows_buffer_words(m, d, world), dtype=torch.int32, device=self.device)
+        rows32 = torch.empty(rows_buffer_words(m, d), dtype=torch.int32, device=self.device)
         j0, j1 = task_range(m, world, rank)
         self.ctx.set_max_level(max_level)
         if j1 > j0:
             self.ctx.mdmc(rows32.data_ptr(), j0, j1, 0, sp)
         rec("t3")
-        exchange_rows(rows32, m, d, self.group)
-        out = {"n_ext": m, "rows32": rows32}
+        out = {"n_ext": m, "rows32": rows32, "shard": (j0, j1)}
         ext_ids = torch.empty(max(m, 1), dtype=torch.int32, device=self.device)
-        mem = torch.empty((n, W), dtype=torch.int32, device=self.device) if membership else None
-        self.ctx.compact(rows32.data_ptr(), mem.data_ptr() if mem is not None else 0, ext_ids.data_ptr(), 0, 0, sp)
+        self.ctx.compact(rows32.data_ptr(), 0, ext_ids.data_ptr(), 0, 0, sp)
         out["ext_ids"] = ext_ids[:m]
+        mem = out_membership
+        if mem is None and membership:
+            mem = torch.empty((n, W), dtype=torch.int32, device=self.device)
+        if mem is not None:
+            if world == 1:
+                if mem.is_cuda:
+                    self.ctx.compact(rows32.data_ptr(), mem.data_ptr(), 0, 0, 0, sp)
+                else:
+                    self.ctx.membership(rows32.data_ptr(), 0, m, 0, n, mem.data_ptr(), sp)
+            else:
+                lo, hi = id_slice(n, world, rank)
+                self.ctx.membership(rows32.data_ptr(), j0, j1, lo, hi, mem.data_ptr(), sp)
         out["membership"] = mem
         if lists:
-            offsets = torch.empty((1 << d) + 1, dtype=torch.int64, device=self.device)
-            total = self.ctx.compact(rows32.data_ptr(), 0, 0, offsets.data_ptr(), 0, sp)
-            ids = torch.empty(max(total, 1), dtype=torch.int32, device=self.device)
-            self.ctx.compact(rows32.data_ptr(), 0, 0, offsets.data_ptr(), ids.data_ptr(), sp)
+            totals = torch.empty(nsub, dtype=torch.int64, device=self.device)
+            self.ctx.lattice_count(rows32.data_ptr(), j0, j1, totals.data_ptr(), sp)
+            all_totals = exchange_totals(totals, self.group)
+            offsets = torch.empty(nsub + 1, dtype=torch.int64, device=self.device)
+            total = self.ctx.lattice_scatter(rows32.data_ptr(), j0, j1, all_totals.data_ptr(), world, rank,
+                                             offsets.data_ptr(), 0, sp)
+            ids = out_ids if out_ids is not None else torch.empty(max(total, 1), dtype=torch.int32, device=self.device)
+            assert ids.numel() >= total, "out_ids too small"
+            self.ctx.lattice_scatter(rows32.data_ptr(), j0, j1, all_totals.data_ptr(), world, rank, 0,
+                                     ids.data_ptr(), sp)
             out["offsets"] = offsets
             out["ids"] = ids[:total]
             out["total_ids"] = total
         if hashcube_w:
+            gather_rows(rows32, m, d, self.group)
             nw, nk, ni = self.ctx.hashcube(rows32.data_ptr(), hashcube_w, sp)
             hc = {"word_offsets": torch.empty(nw + 1, dtype=torch.int64, device=self.device),
                   "keys": torch.empty(max(nk, 1), dtype=torch.int32, device=self.device),

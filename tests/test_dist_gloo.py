@@ -1,8 +1,14 @@
 """Multi-rank sharding and exchange logic of pipeline.py on CPU (gloo, world_size 2 and 3).
 
-The per-rank kernel outputs are stood in by the CPU oracle (test infrastructure), written into exactly
-the buffers and ranges the GPU path writes; the real exchange code (pipeline.exchange_ext /
-exchange_rows) then has to reassemble the full single-rank answer byte for byte.
+The per-rank kernel outputs are stood in by the CPU oracle (test infrastructure), computed for exactly the
+ranges the GPU path gives each rank; the real exchange code (pipeline.exchange_ext / exchange_totals /
+gather_rows) then has to make the distributed result the single-rank answer:
+  * the S+ flags every rank installs equal the full S+ (exchange_ext);
+  * the task ranges tile S+ in rank order, so each subspace's global list is the rank-major concatenation of
+    the ranks' lists and a rank's segment of subspace delta starts at offsets[delta] + the counts of the
+    ranks before it (the placement the lattice scatter kernel performs, from the gathered totals);
+  * the id slices tile [0, n), so every membership row is written by exactly one rank;
+  * gather_rows reassembles the tiled row buffer the HashCube needs.
 """
 from __future__ import annotations
 
@@ -46,14 +52,24 @@ def _tiled(rows_by_j, m, d, nwords):
     return out
 
 
+def _counts(rows, d):
+    """Per-subspace member counts of a set of membership rows."""
+    nsub = 1 << d
+    bits = np.zeros(nsub, np.int64)
+    for delta in range(1, nsub):
+        bits[delta] = int(((rows[:, delta >> 5] >> np.uint32(delta & 31)) & 1).sum())
+    return bits
+
+
 def _worker(rank, world, port, x, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         n, d = x.shape
+        nsub = 1 << d
         order = _key_order(x)
         ext_full = oracle.ext_full(x)
-        # --- K1 stand-in: this rank's tiles of sorted positions
+        # --- K1 stand-in: this rank's blocks of sorted positions
         ext8 = torch.zeros(n, dtype=torch.uint8)
         off, step = pl.prefilter_assignment(rank, world)
         nblk = (n + pl.PREFILTER_BLOCK - 1) // pl.PREFILTER_BLOCK
@@ -64,18 +80,20 @@ def _worker(rank, world, port, x, q):
         flags_sorted = ext8.numpy().astype(bool)
         ext_ids = np.sort(order[flags_sorted])
         m = len(ext_ids)
-        # --- K3 stand-in: rows of this rank's task range, tiled layout, global offsets
+        # --- K3 stand-in: the rows of this rank's task range, in the tiled layout
         rows = oracle.rows_b(x)
-        nwords = pl.rows_buffer_words(m, d, world)
-        buf = np.zeros(nwords, np.uint32)
         j0, j1 = pl.task_range(m, world, rank)
-        assert j0 % 32 == 0 or j0 == j1
-        part = _tiled(np.where(np.arange(m)[:, None] >= j0, rows[ext_ids], 0) * (np.arange(m)[:, None] < j1),
-                      m, d, nwords)
-        buf[:] = part
-        rows32 = torch.from_numpy(buf.view(np.int32).copy())
-        pl.exchange_rows(rows32, m, d)
-        q.put((rank, flags_sorted, ext_ids, rows32.numpy().view(np.uint32).copy(), (j0, j1)))
+        nwords = pl.rows_buffer_words(m, d)
+        mine = np.zeros((m, words_per_row(d)), np.uint32)
+        mine[j0:j1] = rows[ext_ids[j0:j1]]
+        rows32 = torch.from_numpy(_tiled(mine, m, d, nwords).view(np.int32).copy())
+        # --- K4 count stand-in: this rank's per-subspace totals; the real exchange gathers them
+        totals = torch.from_numpy(_counts(rows[ext_ids[j0:j1]], d))
+        all_totals = pl.exchange_totals(totals).numpy().reshape(world, nsub)
+        # --- HashCube path: reassemble the tiled rows
+        pl.gather_rows(rows32, m, d)
+        q.put((rank, ext_ids, (j0, j1), all_totals, rows32.numpy().view(np.uint32).copy(),
+               pl.id_slice(n, world, rank)))
     finally:
         dist.destroy_process_group()
 
@@ -94,26 +112,49 @@ def test_sharded_exchange_reassembles_single_rank_result(world, dist_name, n, d)
         p.join(timeout=60)
         assert p.exitcode == 0
     res.sort(key=lambda t: t[0])
-    # single-rank reference: full oracle rows in the tiled layout
+    nsub = 1 << d
     rows = oracle.rows_b(x)
     ext_ids = np.nonzero(oracle.ext_full(x))[0]
     m = len(ext_ids)
-    want = _tiled(rows[ext_ids], m, d, pl.rows_buffer_words(m, d, world))
-    ranges = [r[4] for r in res]
+    off, ids = oracle.lattice(rows, d)
+    # S+ agreed on every rank; task ranges tile [0, m) in rank order; id slices tile [0, n)
+    ranges = [r[2] for r in res]
     assert ranges[0][0] == 0 and ranges[-1][1] == m
     assert all(ranges[i][1] == ranges[i + 1][0] for i in range(world - 1))
-    for rank, flags, eids, rows32, _ in res:
+    slices = [r[5] for r in res]
+    assert slices[0][0] == 0 and slices[-1][1] == n and all(slices[i][1] == slices[i + 1][0] for i in range(world - 1))
+    for rank, eids, _, all_totals, rows32, _ in res:
         assert np.array_equal(eids, ext_ids)
-        assert np.array_equal(rows32, want), rank
+        # gathered totals: rank-major, and their sum is the global count of every subspace
+        assert np.array_equal(all_totals.sum(axis=0)[1:], np.diff(off)[1:])
+        # the placement: rank r's ids of delta are the global list's slice after the earlier ranks' counts
+        for delta in range(1, nsub):
+            lst = ids[off[delta]:off[delta + 1]]
+            pos = off[delta]
+            for r in range(world):
+                a, b = ranges[r]
+                seg = ids[pos:pos + all_totals[r, delta]]
+                want = np.array([p for p in ext_ids[a:b] if (rows[p, delta >> 5] >> (delta & 31)) & 1], np.int32)
+                assert np.array_equal(seg, want), (rank, r, delta)
+                pos += all_totals[r, delta]
+            assert pos == off[delta + 1] and np.all(np.diff(lst) > 0)
+        # the HashCube path's row gather reassembles the full tiled buffer
+        assert np.array_equal(rows32, _tiled(rows[ext_ids], m, d, pl.rows_buffer_words(m, d))), rank
 
 
 def test_sharding_arithmetic():
     for m in [0, 1, 31, 32, 33, 1000, 123457]:
         for world in [1, 2, 3, 8]:
             rs = [pl.task_range(m, world, r) for r in range(world)]
-            covered = sum(b - a for a, b in rs)
-            assert covered == m
-            for a, b in rs:
+            assert sum(b - a for a, b in rs) == m
+            assert rs[0][0] == 0 and rs[-1][1] == m
+            for i, (a, b) in enumerate(rs):
                 assert a <= b and (a % 32 == 0 or a == b == m)
-            if m:
-                assert pl.chunk_words(m, 12, world) * world <= pl.rows_buffer_words(m, 12, world)
+                if i:
+                    assert rs[i - 1][1] == a
+            groups = [(b - a + 31) // 32 for a, b in rs]
+            assert max(groups) - min(groups) <= 1 or m == 0
+    for n in [0, 1, 7, 1000, 581012]:
+        for world in [1, 2, 3, 8]:
+            sl = [pl.id_slice(n, world, r) for r in range(world)]
+            assert sl[0][0] == 0 and sl[-1][1] == n and all(sl[i][1] == sl[i + 1][0] for i in range(world - 1))

@@ -1,11 +1,12 @@
 // intpeak.cu — integer-pipe peak microbenchmark on one B200 ("Measure with the
 // microbenchmark ... Do not assume 64 vs 128").  The denominators of bench.py's K3 roofline come from here.
 //
-// Three kernels, each a loop of independent dependency chains (8 per thread, 32 warps per SM so the 4-cycle
+// Four kernels, each a loop of independent dependency chains (8 per thread, 32 warps per SM so the 4-cycle
 // fixed latency is hidden), with every operand another chain's value (no constant folding, no hoisting):
 //   alu   LOP3 (majority / mux LUTs: not reassociable), IADD3, PRMT, SHF   -> the ALU pipe only
 //   fma   IMAD (mad.lo.u32)                                                 -> the FMA pipe only
-//   mix   half ALU, half IMAD, interleaved                                  -> both pipes (issue-bound)
+//   mix   half ALU, half IMAD, interleaved, 3 register sources per op       -> both pipes
+//   mix2  the same with 2 register sources + an immediate per op            -> both pipes (issue-bound)
 // Reported: lane-ops per second (CUDA events) and lane-ops per SM per clock (clock64 in every CTA), plus the
 // SM clock during the run derived from the two.  cuobjdump -sass of this file shows the loop bodies
 // (tools/intpeak_sass.txt); every counted op is one SASS instruction.
@@ -51,6 +52,16 @@ __device__ __forceinline__ uint32_t shf(uint32_t a, uint32_t b, uint32_t c) {
     asm volatile("shf.l.wrap.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
     return r;
 }
+__device__ __forceinline__ uint32_t lop_i(uint32_t a, uint32_t b) {  // two register operands + immediate
+    uint32_t r;
+    asm volatile("lop3.b32 %0, %1, %2, 0x5a5a5a5a, 0xE8;" : "=r"(r) : "r"(a), "r"(b));
+    return r;
+}
+__device__ __forceinline__ uint32_t imad_i(uint32_t a, uint32_t c) {  // a * imm + c
+    uint32_t r;
+    asm volatile("mad.lo.u32 %0, %1, 0x9e3779b1, %2;" : "=r"(r) : "r"(a), "r"(c));
+    return r;
+}
 __device__ __forceinline__ uint32_t imad(uint32_t a, uint32_t b, uint32_t c) {
     uint32_t r;
     asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
@@ -59,7 +70,7 @@ __device__ __forceinline__ uint32_t imad(uint32_t a, uint32_t b, uint32_t c) {
 
 constexpr int kChains = 8;
 
-// MODE 0 = alu, 1 = fma, 2 = mix.  Per iteration every chain does 4 ops -> 32 ops per thread per iteration.
+// MODE 0 = alu, 1 = fma, 2 = mix, 3 = mix2.  Per iteration every chain does 4 ops -> 32 ops per thread per iteration.
 template <int MODE>
 __global__ void __launch_bounds__(1024, 1) intpeak_kernel(int iters, uint32_t seed, uint32_t *out,
                                                           unsigned long long *cycles) {
@@ -83,11 +94,16 @@ __global__ void __launch_bounds__(1024, 1) intpeak_kernel(int iters, uint32_t se
                 x = imad(x, c, b);
                 x = imad(x, b, c);
                 x = imad(x, c, b);
-            } else {
+            } else if (MODE == 2) {
                 x = mux(x, b, c);
                 x = imad(x, b, c);
                 x = maj(x, c, b);
                 x = imad(x, c, b);
+            } else {
+                x = lop_i(x, b);
+                x = imad_i(x, c);
+                x = lop_i(x, c);
+                x = imad_i(x, b);
             }
             a[k] = x;
         }
@@ -144,17 +160,20 @@ int main(int argc, char **argv) {
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     cudaDeviceProp prop;
     CK(cudaGetDeviceProperties(&prop, dev));
-    double l[3], f[3], r[3];
+    double l[4], f[4], r[4];
     r[0] = run<0>(iters, sms, &l[0], &f[0]);
     r[1] = run<1>(iters, sms, &l[1], &f[1]);
     r[2] = run<2>(iters, sms, &l[2], &f[2]);
+    r[3] = run<3>(iters, sms, &l[3], &f[3]);
     printf("{\"gpu\": \"%s\", \"sms\": %d, \"iters\": %d, \"threads_per_sm\": 1024, \"chains_per_thread\": %d,\n",
            prop.name, sms, iters, kChains);
-    const char *names[3] = {"alu", "fma", "mix"};
-    const char *what[3] = {"LOP3/IADD3/PRMT/SHF (ALU pipe)", "IMAD (FMA pipe)", "LOP3 + IMAD interleaved (ALU+FMA)"};
-    for (int k = 0; k < 3; k++)
+    const char *names[4] = {"alu", "fma", "mix", "mix2"};
+    const char *what[4] = {"LOP3/IADD3/PRMT/SHF (ALU pipe)", "IMAD (FMA pipe)",
+                           "LOP3 + IMAD interleaved, three register sources each (ALU+FMA)",
+                           "LOP3 + IMAD interleaved, two register sources + an immediate each (ALU+FMA)"};
+    for (int k = 0; k < 4; k++)
         printf(" \"%s\": {\"what\": \"%s\", \"lane_ops_per_s\": %.6e, \"lane_ops_per_sm_per_clk\": %.2f, \"sm_mhz\": %.0f}%s\n",
-               names[k], what[k], r[k], l[k], f[k], k < 2 ? "," : "");
+               names[k], what[k], r[k], l[k], f[k], k < 3 ? "," : "");
     printf("}\n");
     return 0;
 }
