@@ -157,7 +157,8 @@ const char *skycube_last_error(void);   /* thread-local detail of the last error
 
 /* Process-wide tuning / test overrides (performance only: every setting gives the same output bytes).
  * Keys: "k3_design" ('A', 'O' or 0 = automatic), "k3_tpc" (K3 tasks per CTA, 0 = automatic), "k3_mode"
- * (K3 state mode 0/1/2, -1 = automatic), "share_devices" (1: num_gpus ranks may share devices, so the
+ * (K3 state mode 0/1/2, -1 = automatic), "k3_warps" (K3 design A consumer warps: 0 = 16, or 24 at d = 12),
+ * "share_devices" (1: num_gpus ranks may share devices, so the
  * multi-GPU logic can be tested on one GPU), "reset" (all automatic).  EINVAL for an unknown key or value.
  * Serialised with the build calls. */
 skycube_status skycube_set_tuning(const char *key, int32_t value);

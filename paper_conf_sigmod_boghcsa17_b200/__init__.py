@@ -129,7 +129,7 @@ def lib():
         _lib = L
         # tools/*.sh A/B runs name tuning overrides in the environment; applied once, here, never in the
         # library's launch path
-        for key, env in (("k3_design", "SKYCUBE_K3_DESIGN"), ("k3_tpc", "SKYCUBE_K3_TPC"),
+        for key, env in (("k3_design", "SKYCUBE_K3_DESIGN"), ("k3_tpc", "SKYCUBE_K3_TPC"), ("k3_warps", "SKYCUBE_K3_WARPS"),
                          ("k3_mode", "SKYCUBE_K3_MODE"), ("share_devices", "SKYCUBE_SHARE_DEVICES")):
             v = os.environ.get(env, "")
             if v:

@@ -454,6 +454,9 @@ skycube_status skycube_set_tuning(const char *key, int32_t value) {
     } else if (k == "k3_tpc") {
         if (value < 0) return fail(SKYCUBE_EINVAL, "k3_tpc must be >= 0");
         t.k3_tpc = value;
+    } else if (k == "k3_warps") {
+        if (value != 0 && value != 16 && value != 24) return fail(SKYCUBE_EINVAL, "k3_warps must be 0, 16 or 24");
+        t.k3_warps = value;
     } else if (k == "k3_mode") {
         if (value < -1 || value > 2) return fail(SKYCUBE_EINVAL, "k3_mode must be in [-1, 2]");
         t.k3_mode = value;

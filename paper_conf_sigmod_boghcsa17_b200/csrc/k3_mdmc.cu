@@ -73,21 +73,21 @@ constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");
 
-template <int D, int MODE>
+template <int D, int MODE, int NW = kWarps>
 struct GeoK3 {
     static constexpr int PER = (MODE == kModeGlobalTie ? 1 : MODE == kModeSmemTie ? 2 : D + 1) * Geo<D>::WB;
     static constexpr int PS = PER | 1;                                   // odd task stride (bank spread)
     static constexpr int CWP = Geo<D>::CW | 1;                           // odd code stride (box pass)
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
     static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
-    static constexpr int TW = kWarps * REC;                              // tile words
-    static constexpr int kStages = k3_stages<D>();
+    static constexpr int TW = NW * REC;                                  // tile words (one chunk per consumer warp)
+    static constexpr int kStages = NW > kWarps && D < 15 ? 3 : k3_stages<D>();
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
     static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
     static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
-    static constexpr int NT0 = (kSmemBytes / 4 - RING - kWarps * QW - 64) / ROW;
+    static constexpr int NT0 = (kSmemBytes / 4 - RING - NW * QW - 64) / ROW;
     static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                   // tasks per CTA
-    static size_t smem_bytes(int tpc) { return sizeof(uint32_t) * ((size_t)RING + (size_t)tpc * ROW + kWarps * QW); }
+    static size_t smem_bytes(int tpc) { return sizeof(uint32_t) * ((size_t)RING + (size_t)tpc * ROW + NW * QW); }
 };
 
 // Mask of guard bits -> d-bit mask, dimension i -> bit i.  Word k holds dimensions 2k (bits 0-15) and
@@ -148,73 +148,6 @@ __device__ __forceinline__ void exact_masks(const uint32_t *ph, const uint32_t *
     }
 }
 
-// Warp-cooperative walk over the state words whose word index is a subset of H: the lanes take the
-// subsets of the lowest five bits of H, each lane iterates the subsets of the remaining bits.
-template <class F>
-__device__ __forceinline__ void coop_words(uint32_t H, int lane, F &&f) {
-    uint32_t rest = H, w_lo = 0;
-    int np = 0;
-#pragma unroll
-    for (int i = 0; i < 5; i++) {
-        if (rest) {
-            const uint32_t bit = rest & (0u - rest);
-            rest &= rest - 1;
-            if ((lane >> i) & 1) w_lo |= bit;
-            np++;
-        }
-    }
-    if (lane < (1 << np)) {
-        uint32_t w_hi = 0;
-        do {
-            f(w_lo | w_hi);
-            w_hi = (w_hi - rest) & rest;
-        } while (w_hi);
-    }
-    __syncwarp();
-}
-
-// Alg. 3 line 12 for one contributing competitor (S != 0), the whole warp: state st of the task, L and S
-// exact.  Atomic ORs: other warps update the same task concurrently.
-template <int D, int MODE>
-__device__ __forceinline__ void expand(uint32_t *st, uint32_t *tr, int trs, uint32_t L, uint32_t S, uint32_t z,
-                                       int lane) {
-    using G = Geo<D>;
-    const uint32_t lh = L >> 5, lb = sub5(L & 31u);
-    if (MODE == kModeDims) {
-        bool changed = false;  // warp-uniform
-        for (uint32_t s = S; s; s &= s - 1) {  // D_i |= sub(L) for every i in S
-            uint32_t *Di = st + (1 + (__ffs(s) - 1)) * G::WB;
-            if ((Di[lh] >> (L & 31)) & 1u) continue;  // downward closed: sub(L) already there
-            changed = true;
-            coop_words(lh, lane, [&](uint32_t w) { atomicOr(&Di[w], lb); });
-        }
-        if (!changed) return;
-        // K on the words of sub(L) (only there can D change).  Racing warps may compute K from stale D words:
-        // that only leaves K smaller (still sound); bits are only ever OR-ed in.
-        const volatile uint32_t *vs = st;
-        coop_words(lh, lane, [&](uint32_t w) {
-            uint32_t k = 0xffffffffu;
-#pragma unroll
-            for (int i = 0; i < D; i++)
-                if (!((z >> i) & 1u)) k &= vs[(1 + i) * G::WB + w] | ~dim_in_word(i, w);
-            atomicOr(&st[w], k);
-        });
-        return;
-    }
-    // B_{p notin S+} |= sub(S) (strict dominance propagates, L330), unless already there
-    if (!((st[S >> 5] >> (S & 31)) & 1u)) {
-        const uint32_t sb = sub5(S & 31u);
-        coop_words(S >> 5, lane, [&](uint32_t w) { atomicOr(&st[w], sb); });
-    }
-    if (L == S) return;
-    // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}  (reading Q3)
-    const uint32_t E = L & ~S, eh = E >> 5, eb = sub5(E & 31u);
-    coop_words(lh, lane, [&](uint32_t w) {
-        const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
-        if (bits) atomicOr(&tr[w * trs], bits);
-    });
-}
-
 // Shared-memory word access through a 32-bit shared-window address computed once per kernel.  Plain
 // pointer accesses made the compiler re-materialise the dynamic shared base (S2UR SR_CgaCtaId + ULEA) in
 // the hot loops.  Probes are volatile: other warps OR bits into the state concurrently (any value read
@@ -230,6 +163,90 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p) {
     uint32_t a = (uint32_t)__cvta_generic_to_shared(p);
     asm volatile("mov.b32 %0, %0;" : "+r"(a));
     return a;
+}
+
+__device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) { asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+
+// Warp-cooperative walk over the state words whose word index w (the subspace's dimensions 5..d-1) is a subset
+// of H.  Up to 8 words per lane (d <= 13): every lane tests its words w = lane + 32k directly (no subset
+// arithmetic, no loop-carried state; C5 K3 29.5 -> 26.8 ms, C3A 39.4 -> 38.9).  Above (up to 2048 words): the
+// lanes take the subsets of the lowest five set bits of H (the lane index deposited into them), each lane
+// walks the subsets of the remaining bits -- all 32 lanes busy whatever H is.  (A fixed split -- lane = the
+// low five bits of w -- leaves most lanes idle when H has few low bits: C4 K3 660 -> 702 ms.)
+template <int WB, class F>
+__device__ __forceinline__ void coop_words(uint32_t H, int lane, F &&f) {
+    if constexpr (WB <= 256) {
+#pragma unroll
+        for (int k = 0; k < (WB + 31) / 32; k++) {
+            const uint32_t w = (uint32_t)lane + 32u * k;
+            if ((WB % 32 == 0 || w < (uint32_t)WB) && (w & ~H) == 0u) f(w);
+        }
+    } else {
+        uint32_t rest = H, w_lo = 0;
+        int np = 0;
+#pragma unroll
+        for (int i = 0; i < 5; i++) {
+            if (rest) {
+                const uint32_t bit = rest & (0u - rest);
+                rest &= rest - 1;
+                if ((lane >> i) & 1) w_lo |= bit;
+                np++;
+            }
+        }
+        if (lane < (1 << np)) {
+            uint32_t w_hi = 0;
+            do {
+                f(w_lo | w_hi);
+                w_hi = (w_hi - rest) & rest;
+            } while (w_hi);
+        }
+    }
+    __syncwarp();
+}
+
+// Alg. 3 line 12 for one contributing competitor (S != 0), the whole warp: st_s = shared address of the task's
+// state, L and S exact; tie_g = the task's global tie row (kModeGlobalTie, word stride 32), else unused.
+// Atomic ORs (red.shared / red.global): other warps update the same task concurrently.
+template <int D, int MODE>
+__device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t L, uint32_t S, uint32_t z, int lane) {
+    using G = Geo<D>;
+    constexpr int WB = G::WB;
+    const uint32_t lh = L >> 5, lb = sub5(L & 31u);
+    if (MODE == kModeDims) {
+        bool changed = false;  // warp-uniform
+        for (uint32_t s = S; s; s &= s - 1) {  // D_i |= sub(L) for every i in S
+            const uint32_t Di = st_s + 4u * (1 + (__ffs(s) - 1)) * WB;
+            if ((lds_u32(Di + 4u * lh) >> (L & 31)) & 1u) continue;  // downward closed: sub(L) already there
+            changed = true;
+            coop_words<WB>(lh, lane, [&](uint32_t w) { red_or_s(Di + 4u * w, lb); });
+        }
+        if (!changed) return;
+        // K on the words of sub(L) (only there can D change).  Racing warps may compute K from stale D words:
+        // that only leaves K smaller (still sound); bits are only ever OR-ed in.
+        coop_words<WB>(lh, lane, [&](uint32_t w) {
+            uint32_t k = 0xffffffffu;
+#pragma unroll
+            for (int i = 0; i < D; i++)
+                if (!((z >> i) & 1u)) k &= lds_u32(st_s + 4u * ((1 + i) * WB + w)) | ~dim_in_word(i, w);
+            red_or_s(st_s + 4u * w, k);
+        });
+        return;
+    }
+    // B_{p notin S+} |= sub(S) (strict dominance propagates, L330), unless already there
+    if (!((lds_u32(st_s + 4u * (S >> 5)) >> (S & 31)) & 1u)) {
+        const uint32_t sb = sub5(S & 31u);
+        coop_words<WB>(S >> 5, lane, [&](uint32_t w) { red_or_s(st_s + 4u * w, sb); });
+    }
+    if (L == S) return;
+    // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}  (reading Q3)
+    const uint32_t E = L & ~S, eh = E >> 5, eb = sub5(E & 31u);
+    coop_words<WB>(lh, lane, [&](uint32_t w) {
+        const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
+        if (bits) {
+            if (MODE == kModeSmemTie) red_or_s(st_s + 4u * (WB + w), bits);
+            else atomicOr(&tie_g[w * 32], bits);
+        }
+    });
 }
 
 // Partial skycube (Appendix A.2; reading P1): bits b of a membership word whose subspace
@@ -274,7 +291,7 @@ __device__ __forceinline__ void load_row_s(uint32_t a, uint32_t *w) {
 
 // Epilogue of both K3 designs: B_{p notin S} -> membership row (its complement; bit 0, the empty subspace,
 // is never a member), written in the tiled layout (group of 32 tasks, word-major).
-template <int D, int MODE>
+template <int D, int MODE, int NW = kWarps>
 __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, int nt, int warp, int lane, int max_level,
                                            uint32_t *__restrict__ rows32, const uint32_t *__restrict__ tie32,
                                            uint32_t *__restrict__ ext_rows32, uint32_t *__restrict__ host_mem,
@@ -282,7 +299,7 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
     constexpr bool TIES = MODE == kModeSmemTie;
-    for (int t = warp; t < nt; t += kWarps) {
+    for (int t = warp; t < nt; t += NW) {
         const int64_t jt = j0 + t;
         const uint32_t *st = state + t * C::PS;
         uint32_t *out = rows32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
@@ -313,16 +330,15 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
     }
 }
 
-template <int D, int MODE>
-__global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
+template <int D, int MODE, int NW>
+__global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
     int64_t j_end, uint32_t inexact, int tpc, int max_level, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
     uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters, uint32_t *__restrict__ host_mem,
     const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
-    using C = GeoK3<D, MODE>;
-    constexpr bool TIES = MODE == kModeSmemTie;
+    using C = GeoK3<D, MODE, NW>;
     constexpr int CWP = C::CWP, CWV = C::CWV, REC = C::REC;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
@@ -338,9 +354,9 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t st_s = smem_addr(state), wq_s = smem_addr(wq), iq_s = smem_addr(iq), pV_s = smem_addr(pV);
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
-    const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
+    const int64_t ntiles = ceil_div_dev(nchunks, NW);
 
-    if (threadIdx.x == 0) ring.init(kWarps);
+    if (threadIdx.x == 0) ring.init(NW);
     for (int i = threadIdx.x; i < tpc * G::CW; i += blockDim.x) {
         const int t = i / G::CW, k = i % G::CW;
         uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
@@ -368,7 +384,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) state[i] = (i % C::PS) == 0 ? 1u : 0u;
     }
     __syncthreads();
-    if (warp == kWarps) {  // producer warp: one elected lane streams chunk tiles with TMA
+    if (warp == NW) {  // producer warp: one elected lane streams chunk tiles with TMA
         if (lane == 0)
             for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
         return;
@@ -393,7 +409,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
         __threadfence_block();
         __syncwarp();
         if (lane == 0) ring.release(tile);
-        const int64_t c = tile * kWarps + warp;
+        const int64_t c = tile * NW + warp;
         if (c >= nchunks) continue;
 
         // pair pass over packed items (task t, sub-chunk s): lane (k, r) = item k, member r of sub-chunk s; the
@@ -416,8 +432,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             if (miss) {
                 n_miss++;
                 exact_masks<D>(pH + t * CWP, qq, M, inexact, q_ord + (c * 32 + src) * D, p_ord + (j0 + t) * D, L, S);
-                const uint32_t *st = state + t * C::PS;
-                if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
+                if (S != 0 && L != M && ((lds_u32(st_s + 4u * (uint32_t)(t * C::PS + (L >> 5))) >> (L & 31)) & 1u))
+                    S = 0;  // exact L covered
             }
             uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
             n_exp += __popc(todo);
@@ -426,10 +442,9 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
                 todo &= todo - 1;
                 const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
                 const int tb = __shfl_sync(0xffffffffu, t, from);
-                uint32_t *st = state + tb * C::PS;
                 const int64_t jt = j0 + tb;
-                uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-                expand<D, MODE>(st, tr, TIES ? 1 : 32, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
+                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31), Lb, Sb,
+                                MODE == kModeDims ? zm[tb] : 0u, lane);
             }
         };
 
@@ -524,8 +539,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_mdmc_kernel(
             atomicAdd(&counters[6], n_exp);
         }
     }
-    consumer_sync(kWarps * 32);
-    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
+    consumer_sync(NW * 32);
+    write_rows<D, MODE, NW>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
 }
 
 
@@ -552,7 +567,6 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     uint32_t *__restrict__ host_mem, const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
-    constexpr bool TIES = MODE == kModeSmemTie;
     constexpr int CWV = C::CWV, REC = C::REC;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
@@ -633,8 +647,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
                 n_miss++;
                 const int64_t qpos = (tile * kWarps + cl) * 32 + m;
                 exact_masks<D>(ph, qq, M, inexact, q_ord + qpos * D, p_ord + (j0 + t) * D, L, S);
-                const uint32_t *st = state + t * C::PS;
-                if (S != 0 && L != M && ((st[L >> 5] >> (L & 31)) & 1u)) S = 0;  // exact L covered
+                if (S != 0 && L != M && ((lds_u32(st_s + 4u * (uint32_t)(t * C::PS + (L >> 5))) >> (L & 31)) & 1u))
+                    S = 0;  // exact L covered
             }
             uint32_t todo = __ballot_sync(0xffffffffu, S != 0);
             n_exp += __popc(todo);
@@ -643,10 +657,9 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
                 todo &= todo - 1;
                 const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
                 const int tb = __shfl_sync(0xffffffffu, t, from);
-                uint32_t *st = state + tb * C::PS;
                 const int64_t jt = j0 + tb;
-                uint32_t *tr = TIES ? st + G::WB : tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31);
-                expand<D, MODE>(st, tr, TIES ? 1 : 32, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
+                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31), Lb, Sb,
+                                MODE == kModeDims ? zm[tb] : 0u, lane);
             }
         };
 
@@ -777,16 +790,11 @@ bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint
     return true;
 }
 
-template <int D, int MODE>
-void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
+template <int D, int MODE, int NW>
+void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
               cudaStream_t st) {
-    using C = GeoK3<D, MODE>;
+    using C = GeoK3<D, MODE, NW>;
     static_assert(C::NT >= 1, "shared memory too small for one task per CTA");
-    // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
-    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
-    const int design = tuning().k3_design;
-    const bool want_o = design ? design == 'O' : MODE == kModeDims;
-    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
     // tasks per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t range = j_end - j_begin;
     int tpc = (int)std::min<int64_t>(C::NT, std::max<int64_t>(32, ceil_div(ceil_div(range, c.num_sms), 32) * 32));
@@ -804,9 +812,9 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     }
     if (tuning().k3_tpc > 0) tpc = std::max(1, std::min<int>(C::NT, tuning().k3_tpc));
     const size_t smem = C::smem_bytes(tpc);
-    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    SKY_CUDA(cudaFuncSetAttribute(k3_mdmc_kernel<D, MODE, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
-    k3_mdmc_kernel<D, MODE><<<blocks, (kWarps + 1) * 32, smem, st>>>(
+    k3_mdmc_kernel<D, MODE, NW><<<blocks, (NW + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
         c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32,
@@ -819,6 +827,24 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
 // (kModeDims, d <= 12) unless B_{p notin S+} itself is requested (ext rows), then kModeSmemTie.  Continuous
 // data at d > 10: ties are rare and go to a global row (kModeGlobalTie).  skycube_set_tuning("k3_mode", m)
 // forces a mode (parity tests of every mode on the same inputs).
+template <int D, int MODE>
+void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
+              cudaStream_t st) {
+    // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
+    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
+    const int design = tuning().k3_design;
+    const bool want_o = design ? design == 'O' : MODE == kModeDims;
+    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
+    // design A: 16 consumer warps (one chunk each per tile).  k3_warps = 24 (d = 12) is the experiment of more
+    // warps per SM sub-partition against K3's fixed-latency ("wait") stalls (72 registers, 3 ring stages):
+    // H 93.9 -> 90.9 ms but C3A 39.4 -> 40.7 ms (profiles/r02_k3_warps_ab.md), so it stays opt-in.  (32
+    // consumer warps + the producer exceed the 1024-thread CTA limit.)
+    if constexpr (D == 12) {
+        if (tuning().k3_warps == 24) return launch_a<D, MODE, 24>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
+    }
+    launch_a<D, MODE, kWarps>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
+}
+
 template <int D>
 void launch(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
             cudaStream_t st) {

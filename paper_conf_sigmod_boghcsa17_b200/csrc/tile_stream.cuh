@@ -10,13 +10,6 @@
 namespace sky {
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
-// the same, laundered through an opaque move so the compiler keeps the 32-bit value instead of re-deriving it
-// from the dynamic shared base at every use
-__device__ __forceinline__ uint32_t smem_u32_opaque(const void *p) {
-    uint32_t a = (uint32_t)__cvta_generic_to_shared(p);
-    asm volatile("mov.b32 %0, %0;" : "+r"(a));
-    return a;
-}
 
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
@@ -50,6 +43,23 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     } while (!done);
 }
 
+// Producer-side wait (the stage the producer refills is S tiles behind the consumers, so its wake-up latency
+// is hidden): try_wait with a suspend-time hint, the hardware deschedules the waiting producer warp instead of
+// letting it poll.  It replaces a nanosleep back-off whose polling loop was ~5% of K3's issued instructions at
+// H (ncu source view); measured: K1 13.1 -> 12.8 ms at H, K3 unchanged.  (Precomputed 32-bit barrier
+// addresses, and the same hint on the consumers' waits, each measured ~2% slower in K3 and were reverted.)
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+    const uint32_t addr = smem_u32(bar);
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(addr), "r"(parity), "r"(200000u)
+            : "memory");
+    } while (!done);
+}
+
 // Double-buffered stream of fixed-size tiles (bytes multiple of 16, 16-B aligned source).
 struct TileStream2 {
     uint64_t *bar;  // [2] in shared memory
@@ -77,48 +87,6 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-// 32-bit shared-window forms (addresses computed once per kernel: a generic -> shared conversion per probe
-// showed up as ~2% of K3's instructions).  (A try_wait with a suspend-time hint instead of the polling below
-// measured 2% slower at H, C3A and C4: the suspended producer resumes late and the ring drains.)
-__device__ __forceinline__ bool mbar_try_wait_s(uint32_t addr, uint32_t parity) {
-    uint32_t done;
-    asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-        : "=r"(done)
-        : "r"(addr), "r"(parity)
-        : "memory");
-    return done != 0;
-}
-__device__ __forceinline__ void mbar_wait_s(uint32_t addr, uint32_t parity) {
-    while (!mbar_try_wait_s(addr, parity)) {
-    }
-}
-// Producer-side wait (the stage the producer wants to refill is S tiles behind the consumers, so its wake-up
-// latency is hidden): try_wait with a suspend-time hint, so the hardware deschedules the waiting producer warp
-// instead of letting it poll.  The nanosleep back-off this replaces returned early most of the time: its
-// polling loop was ~5% of K3's issued instructions at H (r01/r02 ncu source view, tile_stream.cuh:58-60).
-__device__ __forceinline__ void mbar_wait_sleep_s(uint32_t addr, uint32_t parity) {
-    uint32_t done;
-    do {
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(done)
-            : "r"(addr), "r"(parity), "r"(200000u)
-            : "memory");
-    } while (!done);
-}
-__device__ __forceinline__ void mbar_arrive_s(uint32_t addr) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(addr) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx_s(uint32_t addr, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(addr), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s_s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-                 "l"(src), "r"(bytes), "r"(bar)
-                 : "memory");
-}
-
 // S-stage ring of fixed-size tiles with full (TMA complete_tx) and empty (consumer arrival) barriers.
 // Consumers: wait(t), read stage(t), then one arrival per consumer unit on release(t).
 // Producer (one thread): before issuing tile t >= S, waits until tile t-S released its stage.
@@ -128,14 +96,8 @@ struct TileRing {
     uint64_t *empty;  // [S]
     uint32_t *buf;    // [S][tile_words]
     uint32_t tile_words;
-    uint32_t full_s, empty_s, buf_s;  // the same as 32-bit shared-window addresses
-
-    __device__ TileRing(uint64_t *f, uint64_t *e, uint32_t *b, uint32_t tw)
-        : full(f), empty(e), buf(b), tile_words(tw), full_s(smem_u32_opaque(f)), empty_s(smem_u32_opaque(e)),
-          buf_s(smem_u32_opaque(b)) {}
 
     __device__ __forceinline__ uint32_t *stage(int64_t t) const { return buf + (uint32_t)(t % S) * tile_words; }
-    __device__ __forceinline__ uint32_t stage_s(int64_t t) const { return buf_s + 4u * (uint32_t)(t % S) * tile_words; }
     __device__ __forceinline__ void init(uint32_t consumers) const {
         for (int i = 0; i < S; i++) {
             mbar_init(&full[i], 1);
@@ -145,28 +107,38 @@ struct TileRing {
     }
     __device__ __forceinline__ void issue(const uint32_t *src_tiles, int64_t t) const {
         const int s = (int)(t % S);
-        if (t >= S) mbar_wait_sleep_s(empty_s + 8u * s, (uint32_t)(((t / S) - 1) & 1));
+        if (t >= S) mbar_wait_sleep(&empty[s], (uint32_t)(((t / S) - 1) & 1));
         const uint32_t bytes = tile_words * 4u;
-        mbar_arrive_expect_tx_s(full_s + 8u * s, bytes);
-        bulk_g2s_s(buf_s + 4u * (uint32_t)s * tile_words, src_tiles + t * (int64_t)tile_words, bytes, full_s + 8u * s);
+        mbar_arrive_expect_tx(&full[s], bytes);
+        bulk_g2s(buf + (uint32_t)s * tile_words, src_tiles + t * (int64_t)tile_words, bytes, &full[s]);
     }
-    __device__ __forceinline__ void wait(int64_t t) const { mbar_wait_s(full_s + 8u * (uint32_t)(t % S), (uint32_t)((t / S) & 1)); }
-    __device__ __forceinline__ void release(int64_t t) const { mbar_arrive_s(empty_s + 8u * (uint32_t)(t % S)); }
+    // Two-segment tile: words [0, na) from a + t*na, then words [na, na+nb) from b + t*nb (tile_words = na+nb).
+    __device__ __forceinline__ void issue2(const uint32_t *a, uint32_t na, const uint32_t *b, uint32_t nb,
+                                           int64_t t) const {
+        const int s = (int)(t % S);
+        if (t >= S) mbar_wait_sleep(&empty[s], (uint32_t)(((t / S) - 1) & 1));
+        mbar_arrive_expect_tx(&full[s], (na + nb) * 4u);
+        uint32_t *dst = buf + (uint32_t)s * tile_words;
+        bulk_g2s(dst, a + t * (int64_t)na, na * 4u, &full[s]);
+        bulk_g2s(dst + na, b + t * (int64_t)nb, nb * 4u, &full[s]);
+    }
+    __device__ __forceinline__ void wait(int64_t t) const { mbar_wait(&full[t % S], (uint32_t)((t / S) & 1)); }
+    __device__ __forceinline__ void release(int64_t t) const { mbar_arrive(&empty[t % S]); }
 
     // Filtered streams: the producer fills ring slot k (the k-th streamed tile) with source tile t.
     __device__ __forceinline__ void wait_empty(int64_t slot) const {
-        if (slot >= S) mbar_wait_sleep_s(empty_s + 8u * (uint32_t)(slot % S), (uint32_t)(((slot / S) - 1) & 1));
+        if (slot >= S) mbar_wait_sleep(&empty[slot % S], (uint32_t)(((slot / S) - 1) & 1));
     }
     __device__ __forceinline__ void issue2_slot(const uint32_t *a, uint32_t na, const uint32_t *b, uint32_t nb, int64_t t,
                                                 int64_t slot) const {
         const int s = (int)(slot % S);
-        mbar_arrive_expect_tx_s(full_s + 8u * s, (na + nb) * 4u);
-        const uint32_t dst = buf_s + 4u * (uint32_t)s * tile_words;
-        bulk_g2s_s(dst, a + t * (int64_t)na, na * 4u, full_s + 8u * s);
-        bulk_g2s_s(dst + 4u * na, b + t * (int64_t)nb, nb * 4u, full_s + 8u * s);
+        mbar_arrive_expect_tx(&full[s], (na + nb) * 4u);
+        uint32_t *dst = buf + (uint32_t)s * tile_words;
+        bulk_g2s(dst, a + t * (int64_t)na, na * 4u, &full[s]);
+        bulk_g2s(dst + na, b + t * (int64_t)nb, nb * 4u, &full[s]);
     }
     // completes the slot's phase without data (an end-of-stream marker stored in shared memory before it)
-    __device__ __forceinline__ void arrive_full(int64_t slot) const { mbar_arrive_s(full_s + 8u * (uint32_t)(slot % S)); }
+    __device__ __forceinline__ void arrive_full(int64_t slot) const { mbar_arrive(&full[slot % S]); }
 };
 
 // Named barrier 1 over the consumer warps (the producer warp has left the CTA-wide barrier 0).

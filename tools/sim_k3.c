@@ -215,8 +215,8 @@ int main(int argc, char **argv) {
     const int W = D >= 5 ? 1 << (D - 5) : 1;
     long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     long long g_lane_skip = 0, g_warp_free = 0, g_iters = 0, t_warp_free = 0, t_iters = 0;
-    long long box_after_gtile = 0;
-#pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_box, n_sub, n_pair, n_miss, n_exp, g_lane_skip, g_warp_free, g_iters, t_warp_free, t_iters, box_after_gtile)
+    long long box_after_gtile = 0, n_half = 0, n_sub_h = 0;
+#pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_box, n_sub, n_pair, n_miss, n_exp, g_lane_skip, g_warp_free, g_iters, t_warp_free, t_iters, box_after_gtile, n_half, n_sub_h)
     for (int sg = 0; sg < nsample; sg++) {
         const int g = (int)(((long long)sg * 7919 + 13) % ngroups);
         uint32_t *st = calloc((size_t)32 * W, 4), *tie = calloc((size_t)32 * W, 4);
@@ -253,6 +253,21 @@ int main(int argc, char **argv) {
                     uint32_t Mb = 0;
                     for (int i = 0; i < D; i++) Mb |= (uint32_t)((cc[i] >> BOXSHIFT) <= (pc[i] >> BOXSHIFT)) << i;
                     if (bit(sp, Mb)) continue;
+                    int half_open[2] = {1, 1};
+                    if (NSUB == 8) {  /* three-level variant: half corners (16 points) before the sub-corners */
+                        for (int h = 0; h < 2; h++) {
+                            uint16_t hc[16];
+                            for (int i = 0; i < D; i++) {
+                                uint16_t mn = 0x7fff;
+                                for (int s2 = 4 * h; s2 < 4 * h + 4; s2++)
+                                    if (sub[((long)c * NSUB + s2) * D + i] < mn) mn = sub[((long)c * NSUB + s2) * D + i];
+                                hc[i] = mn;
+                            }
+                            n_half++;
+                            half_open[h] = !bit(sp, le_mask(hc, pc));
+                            if (half_open[h]) n_sub_h += 4;
+                        }
+                    }
                     for (int s = 0; s < NSUB; s++) {
                         n_sub++;
                         if (bit(sp, le_mask(sub + ((long)c * NSUB + s) * D, pc))) continue;
@@ -293,6 +308,7 @@ int main(int argc, char **argv) {
            N, D, m, nch, CS, SS, task_order, chunk_order, nsample);
     printf(" \"box\": %.4g, \"sub\": %.4g, \"pair\": %.4g, \"miss\": %.4g, \"expansions\": %.4g,\n", n_box * scale,
            n_sub * scale, n_pair * scale, n_miss * scale, n_exp * scale);
+    printf(" \"three_level\": {\"half\": %.4g, \"sub\": %.4g},\n", n_half * scale, n_sub_h * scale);
     printf(" \"gbox_lane_skip_frac\": %.4f, \"gbox_warp_free_frac\": %.4f, \"gtile_warp_free_frac\": %.4f,"
            " \"box_after_gtile_frac\": %.4f}\n",
            (double)g_lane_skip / n_box, (double)g_warp_free / g_iters, (double)t_warp_free / t_iters,
