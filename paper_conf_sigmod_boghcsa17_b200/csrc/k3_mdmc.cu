@@ -67,8 +67,11 @@ constexpr int kWarps = 16;                // consumer warps = chunks per tile (+
 #ifndef SKY_K3_STAGES
 #define SKY_K3_STAGES 4
 #endif
+#ifndef SKY_K3_STAGES_HIGHD
+#define SKY_K3_STAGES_HIGHD 2
+#endif
 template <int D>
-constexpr int k3_stages() { return D >= 15 ? 2 : SKY_K3_STAGES; }
+constexpr int k3_stages() { return D >= 15 ? SKY_K3_STAGES_HIGHD : SKY_K3_STAGES; }
 constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");

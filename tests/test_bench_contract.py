@@ -42,3 +42,13 @@ def test_reference_arm_nonzero_rank_is_silent():
     r = _run({"RANK": "1", "LOCAL_RANK": "1", "WORLD_SIZE": "2"})
     assert r.returncode == 0, r.stderr[-2000:]
     assert r.stdout.strip() == ""
+
+
+def test_gpus_flag_fails_loudly_without_enough_devices():
+    """`bench.py --gpus N` re-launches itself as N ranks; with fewer than N CUDA devices visible (none here) it
+    must fail with a message instead of silently timing fewer GPUs (n_gpus must equal --gpus)."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1", "--warmup", "0"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode != 0
+    assert "--gpus 2 requested" in r.stderr
+    assert r.stdout.strip() == ""

@@ -1,0 +1,24 @@
+#!/bin/bash
+# GPU-box helper (round 2 final evidence): GPU tests (incl. the full-size digest test), smoke, bench lines
+# for every config (+ HashCube, k3_warps=24 and the reference arm at H), the ncu launch list of the default
+# bench and one --set full capture of K3 at H (kept: tools/evidence_summary.py + traffic.json need it).
+mkdir -p gpurun_out
+rm -f gpurun_out/ev_*
+python -c "from paper_conf_sigmod_boghcsa17_b200 import build; build.build()" || exit 1
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gpurun_out/ev_gpu.txt
+if [ "${TESTS:-1}" = 1 ]; then
+  timeout 1500 python -m pytest tests -m gpu -q 2>&1 | tail -6 > gpurun_out/ev_tests.log
+fi
+python __graft_entry__.py smoke > gpurun_out/ev_smoke.log 2>&1
+for c in ${CONFIGS:-H C3A C3I C3C C2 C5 C4}; do
+  timeout 900 python bench.py --config $c --cpu-seconds ${CPU_S:-8} 2>/dev/null | tail -1 > gpurun_out/ev_bench_$c.json
+done
+timeout 600 python bench.py --output hashcube --cpu-seconds 2 2>/dev/null | tail -1 > gpurun_out/ev_bench_H_hashcube.json
+SKYCUBE_K3_WARPS=24 timeout 600 python bench.py --cpu-seconds 2 --no-e2e 2>/dev/null | tail -1 > gpurun_out/ev_bench_H_warps24.json
+timeout 900 python bench.py --impl reference --steps 2 --warmup 1 2>/dev/null | tail -1 > gpurun_out/ev_bench_H_reference.json
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_launches_H.csv \
+  python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > gpurun_out/ev_ncu_launch.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k3_mdmc -c 1 -f -o gpurun_out/ev_prof_k3_mdmc_H \
+  python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k3_mdmc_H.log 2>&1
+cat gpurun_out/ev_tests.log gpurun_out/ev_smoke.log
+for f in gpurun_out/ev_bench_*.json; do echo "$f: $(head -c 160 $f)"; done

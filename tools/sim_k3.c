@@ -215,8 +215,8 @@ int main(int argc, char **argv) {
     const int W = D >= 5 ? 1 << (D - 5) : 1;
     long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     long long g_lane_skip = 0, g_warp_free = 0, g_iters = 0, t_warp_free = 0, t_iters = 0;
-    long long box_after_gtile = 0, n_half = 0, n_sub_h = 0;
-#pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_box, n_sub, n_pair, n_miss, n_exp, g_lane_skip, g_warp_free, g_iters, t_warp_free, t_iters, box_after_gtile, n_half, n_sub_h)
+    long long box_after_gtile = 0, n_half = 0, n_sub_h = 0, lb_sub = 0, lb_pair = 0, lb_open = 0;
+#pragma omp parallel for schedule(dynamic, 1) reduction(+ : n_box, n_sub, n_pair, n_miss, n_exp, g_lane_skip, g_warp_free, g_iters, t_warp_free, t_iters, box_after_gtile, n_half, n_sub_h, lb_sub, lb_pair, lb_open)
     for (int sg = 0; sg < nsample; sg++) {
         const int g = (int)(((long long)sg * 7919 + 13) % ngroups);
         uint32_t *st = calloc((size_t)32 * W, 4), *tie = calloc((size_t)32 * W, 4);
@@ -300,6 +300,21 @@ int main(int argc, char **argv) {
                 g_warp_free += allg;
             }
         }
+        /* lower bound for any visiting order: the tests a pass with the final (saturated) state still runs */
+        for (int l = 0; l < 32; l++) {
+            uint32_t *sp = st + l * W;
+            const uint16_t *pc = CODE + (long)tasks[g * 32 + l] * D;
+            for (int c = 0; c < nch; c++) {
+                const uint16_t *cc = corner + (long)c * D;
+                if (bit(sp, le_mask(cc, pc))) continue;
+                lb_open++;
+                for (int s2 = 0; s2 < NSUB; s2++) {
+                    lb_sub++;
+                    if (bit(sp, le_mask(sub + ((long)c * NSUB + s2) * D, pc))) continue;
+                    lb_pair += SS;
+                }
+            }
+        }
         free(st);
         free(tie);
     }
@@ -309,6 +324,8 @@ int main(int argc, char **argv) {
     printf(" \"box\": %.4g, \"sub\": %.4g, \"pair\": %.4g, \"miss\": %.4g, \"expansions\": %.4g,\n", n_box * scale,
            n_sub * scale, n_pair * scale, n_miss * scale, n_exp * scale);
     printf(" \"three_level\": {\"half\": %.4g, \"sub\": %.4g},\n", n_half * scale, n_sub_h * scale);
+    printf(" \"saturated_state_lower_bound\": {\"open\": %.4g, \"sub\": %.4g, \"pair\": %.4g},\n", lb_open * scale,
+           lb_sub * scale, lb_pair * scale);
     printf(" \"gbox_lane_skip_frac\": %.4f, \"gbox_warp_free_frac\": %.4f, \"gtile_warp_free_frac\": %.4f,"
            " \"box_after_gtile_frac\": %.4f}\n",
            (double)g_lane_skip / n_box, (double)g_warp_free / g_iters, (double)t_warp_free / t_iters,
