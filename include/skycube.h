@@ -38,7 +38,9 @@ typedef enum {
     SKYCUBE_ENAN = 2,   /* a NaN in the input */
     SKYCUBE_ENOMEM = 3, /* host or device allocation failed */
     SKYCUBE_ECUDA = 4,  /* CUDA runtime / kernel error */
-    SKYCUBE_ENCCL = 5,  /* reserved: collective error (multi-GPU) */
+    SKYCUBE_ENCCL = 5,  /* reserved for a collective-library error; not returned today: the
+                           single-process num_gpus path exchanges with CUDA peer copies (errors: ECUDA) and
+                           the per-rank path leaves collectives to the caller (torch.distributed / NCCL) */
     SKYCUBE_ENODEV = 6  /* no sm_100 device visible */
 } skycube_status;
 
@@ -157,7 +159,7 @@ const char *skycube_last_error(void);   /* thread-local detail of the last error
 
 /* Process-wide tuning / test overrides (performance only: every setting gives the same output bytes).
  * Keys: "k3_design" ('A', 'O' or 0 = automatic), "k3_tpc" (K3 tasks per CTA, 0 = automatic), "k3_mode"
- * (K3 state mode 0/1/2, -1 = automatic), "k3_warps" (K3 design A consumer warps: 0 = 16, or 24 at d = 12),
+ * (K3 state mode 0/1/2, -1 = automatic), "k3_warps" (K3 design A consumer warps: 0 = automatic (24 at d = 12, else 16), 16 forces 16),
  * "share_devices" (1: num_gpus ranks may share devices, so the
  * multi-GPU logic can be tested on one GPU), "reset" (all automatic).  EINVAL for an unknown key or value.
  * Serialised with the build calls. */

@@ -45,7 +45,7 @@ struct Error {
 struct Tuning {
     int k3_design = 0;      // 'A' or 'O': force a K3 design
     int k3_tpc = 0;         // force K3 tasks per CTA (design A)
-    int k3_warps = 0;       // K3 design A consumer warps (16 default; 24 at d = 12: experiment)
+    int k3_warps = 0;       // K3 design A consumer warps: 0 = automatic (24 at d = 12, else 16), or 16 / 24
     int k3_mode = -1;       // force a K3 state mode (0, 1, 2); -1 = automatic
     int share_devices = 0;  // 1: multi-GPU ranks may share devices (tests of the k-rank logic on one GPU)
 };

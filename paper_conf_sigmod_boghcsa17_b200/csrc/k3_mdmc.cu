@@ -169,6 +169,20 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p) {
 }
 
 __device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) { asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+__device__ __forceinline__ void exch_s(uint32_t a, uint32_t v) {
+    uint32_t old;
+    asm volatile("atom.shared.exch.b32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
+}
+
+// kModeGlobalTie: the tie rows are zeroed before the kernel (memset) and a task's row is marked in shared memory
+// (flag 2) when a tie is first OR-ed into it; the epilogue reads only marked rows.  Ties are rare in the
+// continuous data this mode runs on, so the epilogue's read-back of 8 KB per task at d = 16 disappears (C4:
+// 7.3 GB of the 15.4 GB of DRAM traffic per K3 launch in round 1).  (Zeroing the rows lazily in the kernel
+// instead of the memset lost tie bits to a race -- tests/test_gpu_parity.py::test_global_tie_rows_d16 --
+// and was dropped.)
+__device__ __forceinline__ void tie_row_mark(uint32_t flag_s, int lane) {
+    if (lane == 0) exch_s(flag_s, 2u);
+}
 
 // Warp-cooperative walk over the state words whose word index w (the subspace's dimensions 5..d-1) is a subset
 // of H.  Up to 8 words per lane (d <= 13): every lane tests its words w = lane + 32k directly (no subset
@@ -211,7 +225,8 @@ __device__ __forceinline__ void coop_words(uint32_t H, int lane, F &&f) {
 // state, L and S exact; tie_g = the task's global tie row (kModeGlobalTie, word stride 32), else unused.
 // Atomic ORs (red.shared / red.global): other warps update the same task concurrently.
 template <int D, int MODE>
-__device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t L, uint32_t S, uint32_t z, int lane) {
+__device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t tflag_s, uint32_t L, uint32_t S, uint32_t z,
+                                       int lane) {
     using G = Geo<D>;
     constexpr int WB = G::WB;
     const uint32_t lh = L >> 5, lb = sub5(L & 31u);
@@ -243,6 +258,7 @@ __device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t 
     if (L == S) return;
     // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}  (reading Q3)
     const uint32_t E = L & ~S, eh = E >> 5, eb = sub5(E & 31u);
+    if (MODE == kModeGlobalTie) tie_row_mark(tflag_s, lane);
     coop_words<WB>(lh, lane, [&](uint32_t w) {
         const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
         if (bits) {
@@ -298,7 +314,7 @@ template <int D, int MODE, int NW = kWarps>
 __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, int nt, int warp, int lane, int max_level,
                                            uint32_t *__restrict__ rows32, const uint32_t *__restrict__ tie32,
                                            uint32_t *__restrict__ ext_rows32, uint32_t *__restrict__ host_mem,
-                                           const int32_t *__restrict__ ext_ids) {
+                                           const int32_t *__restrict__ ext_ids, const uint32_t *tflag) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE>;
     constexpr bool TIES = MODE == kModeSmemTie;
@@ -310,6 +326,7 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
         // zero-copy: the row also goes straight to the caller's pinned host membership array (by point id),
         // so its PCIe transfer overlaps the rest of the kernel instead of following the whole build
         uint32_t *hrow = host_mem ? host_mem + (int64_t)ext_ids[jt] * G::WB : nullptr;
+        const bool tie_used = MODE == kModeGlobalTie && tflag[t] == 2u;
         for (int w = lane; w < G::WB; w += 32) {
             uint32_t v;
             if (MODE == kModeDims) {  // p dominated in delta <=> delta in D_i for some i in delta
@@ -317,7 +334,8 @@ __device__ __forceinline__ void write_rows(const uint32_t *state, int64_t j0, in
 #pragma unroll
                 for (int i = 0; i < D; i++) v |= st[(1 + i) * G::WB + w] & dim_in_word(i, w);
             } else {
-                v = st[w] | (TIES ? st[G::WB + w] : trg[w * 32]);
+                // tie rows are read from L2 (ld.global.cg): they were written by atomics during this kernel
+                v = st[w] | (TIES ? st[G::WB + w] : tie_used ? __ldcg(&trg[w * 32]) : 0u);
             }
             const uint32_t lvl = max_level > 0 ? level_pattern(max_level - __popc(w)) : 0xffffffffu;
             uint32_t row = ~v & G::kRowMask & lvl;
@@ -355,6 +373,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
     uint32_t *wq = zm + tpc + warp * C::QW;    // per-warp queue of opened tasks (<= 3 + 32 entries)
     uint32_t *iq = wq + 40;                    // per-warp queue of opened (task, sub-chunk) items (<= 7 + 32)
     const uint32_t st_s = smem_addr(state), wq_s = smem_addr(wq), iq_s = smem_addr(iq), pV_s = smem_addr(pV);
+    const uint32_t zm_s = smem_addr(zm);  // kModeGlobalTie: per-task tie-row flags (kModeDims: Z_p)
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
     const int64_t ntiles = ceil_div_dev(nchunks, NW);
@@ -385,6 +404,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
         }
     } else {
         for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) state[i] = (i % C::PS) == 0 ? 1u : 0u;
+        for (int t = threadIdx.x; t < tpc; t += blockDim.x) zm[t] = 0u;  // tie rows untouched
     }
     __syncthreads();
     if (warp == NW) {  // producer warp: one elected lane streams chunk tiles with TMA
@@ -446,8 +466,8 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
                 const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
                 const int tb = __shfl_sync(0xffffffffu, t, from);
                 const int64_t jt = j0 + tb;
-                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31), Lb, Sb,
-                                MODE == kModeDims ? zm[tb] : 0u, lane);
+                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31),
+                                zm_s + 4u * (uint32_t)tb, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
             }
         };
 
@@ -543,7 +563,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
         }
     }
     consumer_sync(NW * 32);
-    write_rows<D, MODE, NW>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
+    write_rows<D, MODE, NW>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids, zm);
 }
 
 
@@ -610,6 +630,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         }
     } else {
         for (int i = threadIdx.x; i < tpc * C::PS; i += blockDim.x) state[i] = (i % C::PS) == 0 ? 1u : 0u;
+        for (int t = threadIdx.x; t < tpc; t += blockDim.x) zm[t] = 0u;  // tie rows untouched
     }
     __syncthreads();
     if (warp == kWarps) {  // producer warp: one elected lane streams chunk tiles with TMA
@@ -618,6 +639,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         return;
     }
     const uint32_t st_s = smem_addr(state), pV_s = smem_addr(pV), q1_s = smem_addr(q1), q2_s = smem_addr(q2);
+    const uint32_t zm_s = smem_addr(zm);  // kModeGlobalTie: per-task tie-row flags (kModeDims: Z_p)
     const uint32_t ring_s = smem_addr(smem + 4 * kStages);
     const int wpg = kWarps / ngrp, grp = warp / wpg, wsub = warp % wpg;
     const int town = grp * 32 + lane;                         // this lane's task
@@ -661,8 +683,8 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
                 const uint32_t Sb = __shfl_sync(0xffffffffu, S, from), Lb = __shfl_sync(0xffffffffu, L, from);
                 const int tb = __shfl_sync(0xffffffffu, t, from);
                 const int64_t jt = j0 + tb;
-                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31), Lb, Sb,
-                                MODE == kModeDims ? zm[tb] : 0u, lane);
+                expand<D, MODE>(st_s + 4u * (uint32_t)(tb * C::PS), tie32 + (jt >> 5) * (G::WB * 32) + (jt & 31),
+                                zm_s + 4u * (uint32_t)tb, Lb, Sb, MODE == kModeDims ? zm[tb] : 0u, lane);
             }
         };
 
@@ -752,7 +774,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         }
     }
     consumer_sync(kWarps * 32);
-    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids);
+    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids, zm);
 }
 
 template <int D, int MODE>
@@ -838,12 +860,13 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     const int design = tuning().k3_design;
     const bool want_o = design ? design == 'O' : MODE == kModeDims;
     if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
-    // design A: 16 consumer warps (one chunk each per tile).  k3_warps = 24 (d = 12) is the experiment of more
-    // warps per SM sub-partition against K3's fixed-latency ("wait") stalls (72 registers, 3 ring stages):
-    // H 93.9 -> 90.9 ms but C3A 39.4 -> 40.7 ms (profiles/r02_k3_warps_ab.md), so it stays opt-in.  (32
-    // consumer warps + the producer exceed the 1024-thread CTA limit.)
+    // design A: one chunk per consumer warp per tile.  At d = 12, 24 consumer warps (72 registers, 3 ring stages
+    // of 24 chunks) instead of 16 (89 registers, 4 stages of 16): more warps per SM sub-partition against K3's
+    // fixed-latency ("wait") stalls.  With the round-2 expansion walk it measured H 94.2 -> 89.5 ms, C3A 39.3 ->
+    // 37.2, C3I 7.6 -> 7.5 (profiles/r02_k3_warps_ab.md), so it is the default there; k3_warps = 16 forces
+    // the 16-warp kernel.  (32 consumer warps + the producer exceed the 1024-thread CTA limit.)
     if constexpr (D == 12) {
-        if (tuning().k3_warps == 24) return launch_a<D, MODE, 24>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
+        if (tuning().k3_warps != 16) return launch_a<D, MODE, 24>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
     }
     launch_a<D, MODE, kWarps>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
 }
@@ -873,10 +896,11 @@ void mdmc_run(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *d_rows32, uint32
     if (!c.ext_ready) throw Error{1, "skycube_dev_mdmc before skycube_dev_set_ext"};
     if (j_begin < 0 || j_end > c.m || (j_begin & 31)) throw Error{1, "bad MDMC task range"};
     if (j_end <= j_begin) return;
-    const int64_t g0 = j_begin >> 5, g1 = ceil_div(j_end, 32);
+    // the tie rows (kModeGlobalTie; the epilogue reads only the rows a tie was OR-ed into)
     const size_t grp_words = (size_t)c.W * 32;
     c.tie.ensure(sizeof(uint32_t) * grp_words * (size_t)ceil_div(c.m, 32));
-    SKY_CUDA(cudaMemsetAsync(c.tie.as<uint32_t>() + g0 * grp_words, 0, sizeof(uint32_t) * grp_words * (g1 - g0), st));
+    SKY_CUDA(cudaMemsetAsync(c.tie.as<uint32_t>() + (j_begin >> 5) * grp_words, 0,
+                             sizeof(uint32_t) * grp_words * (ceil_div(j_end, 32) - (j_begin >> 5)), st));
     switch (c.d) {
 #define SKY_K3(DD) case DD: launch<DD>(c, j_begin, j_end, d_rows32, d_ext_rows32, host_membership, st); break;
         SKY_K3(1) SKY_K3(2) SKY_K3(3) SKY_K3(4) SKY_K3(5) SKY_K3(6) SKY_K3(7) SKY_K3(8)

@@ -240,3 +240,33 @@ def test_k3_designs_and_modes(tuning, design, mode, case):
     assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
     off, ids = oracle.lattice(want, d)
     assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)
+
+
+@pytest.mark.parametrize("warps", [16, 24])
+@pytest.mark.parametrize("mode", ["0", "1"])
+@pytest.mark.parametrize("case", [("A", 7000, 12, 911), ("I", 5000, 12, 912)])
+def test_k3_design_a_warp_counts(tuning, warps, mode, case):
+    """Design A at d = 12 with 16 and with 24 consumer warps (one chunk per warp per tile: tiles of 16 or 24
+    chunks, 4 or 3 ring stages), on several tiles with ragged tails; both must equal the oracle."""
+    tuning("k3_warps", warps)
+    tuning("k3_design", "A")
+    tuning("k3_mode", int(mode))
+    dist, n, d, seed = case
+    x = datagen.generate(dist, n, d, seed)
+    want = oracle.rows_b(x)
+    r = sky.skycube_build(x)
+    bad = np.nonzero((r["rows"] != want).any(axis=1))[0]
+    assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
+
+
+def test_global_tie_rows_d16(tuning):
+    """kModeGlobalTie at d = 16 on tie-heavy data, built three times in a row: the epilogue reads a task's global
+    tie row only if a tie was OR-ed into it (flag in shared memory); every row must still equal the oracle.
+    (A variant that zeroed the rows lazily inside K3 failed this test: lost tie bits.)"""
+    tuning("k3_mode", 0)
+    x = datagen.small_int_grid(433, 16, 3, 4242)
+    want = oracle.rows_b(x)
+    for _ in range(3):
+        r = sky.skycube_build(x)
+        bad = np.nonzero((r["rows"] != want).any(axis=1))[0]
+        assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
