@@ -133,7 +133,7 @@ int64_t sdsc_run(Ctx &c, int64_t *d_offsets, uint32_t *d_membership, cudaStream_
 int64_t hashcube_words(int d, uint32_t w);
 void hashcube_build(Ctx &c, const uint32_t *rows32, uint32_t w, cudaStream_t st);
 
-constexpr int64_t kQPad = 3072;      // competitor stream padded to whole MDMC tiles (16, 24 or 32 chunks)
+constexpr int64_t kQPad = 21504;     // competitor stream padded to whole MDMC tiles (16, 24, 28 or 32 chunks)
 constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk tiles (16 chunks) are whole
 constexpr int kTileChunks = 16;         // chunks per competitor tile (one super-chunk of 512 points)
 constexpr int kSubSize = 4;             // points per sub-chunk (K3 level below the chunk)

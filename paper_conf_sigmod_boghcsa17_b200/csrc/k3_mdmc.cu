@@ -67,6 +67,10 @@ constexpr int kWarps = 16;                // consumer warps = chunks per tile (+
 #ifndef SKY_K3_STAGES
 #define SKY_K3_STAGES 4
 #endif
+#ifndef SKY_K3_STAGES_WIDE
+#define SKY_K3_STAGES_WIDE 2  // ring stages of the 24-warp (24-chunk tile) kernel: 2 measured better than 3
+                              // (C3A K3 35.6 -> 34.0 ms: more tasks per CTA; H 87.1 -> 86.7)
+#endif
 #ifndef SKY_K3_STAGES_HIGHD
 #define SKY_K3_STAGES_HIGHD 2
 #endif
@@ -84,7 +88,7 @@ struct GeoK3 {
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
     static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
     static constexpr int TW = NW * REC;                                  // tile words (one chunk per consumer warp)
-    static constexpr int kStages = NW > kWarps && D < 15 ? 3 : k3_stages<D>();
+    static constexpr int kStages = NW > kWarps && D < 15 ? SKY_K3_STAGES_WIDE : k3_stages<D>();
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
     static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
     static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
@@ -860,11 +864,12 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     const int design = tuning().k3_design;
     const bool want_o = design ? design == 'O' : MODE == kModeDims;
     if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
-    // design A: one chunk per consumer warp per tile.  At d = 12, 24 consumer warps (72 registers, 3 ring stages
+    // design A: one chunk per consumer warp per tile.  At d = 12, 24 consumer warps (70 registers, 2 ring stages
     // of 24 chunks) instead of 16 (89 registers, 4 stages of 16): more warps per SM sub-partition against K3's
     // fixed-latency ("wait") stalls.  With the round-2 expansion walk it measured H 94.2 -> 89.5 ms, C3A 39.3 ->
     // 37.2, C3I 7.6 -> 7.5 (profiles/r02_k3_warps_ab.md), so it is the default there; k3_warps = 16 forces
-    // the 16-warp kernel.  (32 consumer warps + the producer exceed the 1024-thread CTA limit.)
+    // the 16-warp kernel.  (28 warps measured slower: H 87.5-90.6 ms; 32 consumer warps + the producer exceed
+    // the 1024-thread CTA limit.)
     if constexpr (D == 12) {
         if (tuning().k3_warps != 16) return launch_a<D, MODE, 24>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st);
     }
