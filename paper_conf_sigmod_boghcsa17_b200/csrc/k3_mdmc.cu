@@ -80,7 +80,7 @@ constexpr int kSmemBytes = 227 * 1024;    // opt-in maximum per CTA
 constexpr int kModeGlobalTie = 0, kModeSmemTie = 1, kModeDims = 2;
 static_assert(kWarps == kTileChunks, "one chunk per consumer warp per tile");
 
-template <int D, int MODE, int NW = kWarps>
+template <int D, int MODE, int NW = kWarps, int ST = 0>
 struct GeoK3 {
     static constexpr int PER = (MODE == kModeGlobalTie ? 1 : MODE == kModeSmemTie ? 2 : D + 1) * Geo<D>::WB;
     static constexpr int PS = PER | 1;                                   // odd task stride (bank spread)
@@ -88,7 +88,7 @@ struct GeoK3 {
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
     static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
     static constexpr int TW = NW * REC;                                  // tile words (one chunk per consumer warp)
-    static constexpr int kStages = NW > kWarps && D < 15 ? SKY_K3_STAGES_WIDE : k3_stages<D>();
+    static constexpr int kStages = ST > 0 ? ST : NW > kWarps && D < 15 ? SKY_K3_STAGES_WIDE : k3_stages<D>();
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
     static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
     static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
@@ -585,15 +585,20 @@ __device__ __forceinline__ void load_row2_s(uint32_t a, uint32_t *w) {
 // reloads, no per-group loop.  Opened (task, chunk) items are queued and run through the same sub-chunk and
 // pair passes as design A, reading the chunk's sub-corners and competitors from the ring stage, which the
 // warp holds until it has finished the tile.  Needs 32 tasks' state in shared memory (d <= 15).
-template <int D, int MODE>
-__global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
+// design O's ring: 3 stages with 24 warps (a warp holds its stage until its sub/pair passes are done; C5 K3
+// 20.6 ms with 2 stages, 20.2 with 3)
+template <int D, int MODE, int NW>
+using GeoO = GeoK3<D, MODE, NW, (NW > kWarps && D < 15 ? 3 : 0)>;
+
+template <int D, int MODE, int NW>
+__global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
     int64_t j_end, uint32_t inexact, int ngrp, int max_level, uint32_t *__restrict__ rows32,
     uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters,
     uint32_t *__restrict__ host_mem, const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
-    using C = GeoK3<D, MODE>;
+    using C = GeoO<D, MODE, NW>;
     constexpr int CWV = C::CWV, REC = C::REC;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
@@ -608,9 +613,9 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     uint32_t *q2 = q1 + 40;                    // opened (task, chunk, sub-chunk) items (<= 7 + 32)
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
-    const int64_t ntiles = ceil_div_dev(nchunks, kWarps);
+    const int64_t ntiles = ceil_div_dev(nchunks, NW);
 
-    if (threadIdx.x == 0) ring.init(kWarps);
+    if (threadIdx.x == 0) ring.init(NW);
     for (int i = threadIdx.x; i < tpc * G::CW; i += blockDim.x) {
         const int t = i / G::CW, k = i % G::CW;
         uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
@@ -637,7 +642,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         for (int t = threadIdx.x; t < tpc; t += blockDim.x) zm[t] = 0u;  // tie rows untouched
     }
     __syncthreads();
-    if (warp == kWarps) {  // producer warp: one elected lane streams chunk tiles with TMA
+    if (warp == NW) {  // producer warp: one elected lane streams chunk tiles with TMA
         if (lane == 0)
             for (int64_t t = 0; t < ntiles; t++) ring.issue(chunks, t);
         return;
@@ -645,7 +650,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
     const uint32_t st_s = smem_addr(state), pV_s = smem_addr(pV), q1_s = smem_addr(q1), q2_s = smem_addr(q2);
     const uint32_t zm_s = smem_addr(zm);  // kModeGlobalTie: per-task tie-row flags (kModeDims: Z_p)
     const uint32_t ring_s = smem_addr(smem + 4 * kStages);
-    const int wpg = kWarps / ngrp, grp = warp / wpg, wsub = warp % wpg;
+    const int wpg = NW / ngrp, grp = warp / wpg, wsub = warp % wpg;
     const int town = grp * 32 + lane;                         // this lane's task
     const uint32_t valid = __ballot_sync(0xffffffffu, town < nt);
     uint32_t p[G::CW];
@@ -660,7 +665,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         auto pair_pass = [&](int base, int cnt) {
             const int k8 = lane >> 2, r = lane & 3;
             const uint32_t it = lds_u32(q2_s + 4u * (base + min(k8, cnt - 1)));
-            const int t = (int)(it >> 7), cl = (int)((it >> 3) & 15u), sidx = (int)(it & 7u);
+            const int t = (int)(it >> 8), cl = (int)((it >> 3) & 31u), sidx = (int)(it & 7u);  // cl < NW <= 32
             const int m = sidx * kSubSize + r;                       // member of the chunk
             uint32_t qq[G::CW], x[G::CW], ph[G::CW];
             load_row2_s<G::CW>(stg_s + 4u * (cl * REC + m * G::CW), qq);
@@ -674,7 +679,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
             uint32_t L = 0, S = 0;
             if (miss) {
                 n_miss++;
-                const int64_t qpos = (tile * kWarps + cl) * 32 + m;
+                const int64_t qpos = (tile * NW + cl) * 32 + m;
                 exact_masks<D>(ph, qq, M, inexact, q_ord + qpos * D, p_ord + (j0 + t) * D, L, S);
                 if (S != 0 && L != M && ((lds_u32(st_s + 4u * (uint32_t)(t * C::PS + (L >> 5))) >> (L & 31)) & 1u))
                     S = 0;  // exact L covered
@@ -697,7 +702,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         auto sub_pass = [&](int base, int cnt) {
             const int u = lane >> 3, sidx = lane & 7;
             const uint32_t it = lds_u32(q1_s + 4u * (base + min(u, cnt - 1)));
-            const int t = (int)(it >> 4), cl = (int)(it & 15u);
+            const int t = (int)(it >> 5), cl = (int)(it & 31u);
             uint32_t x[G::CW], sc[G::CW];
             load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
             load_row2_s<G::CW>(stg_s + 4u * (cl * REC + (33 + sidx) * G::CW), sc);
@@ -710,7 +715,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
             n_sub += 8 * cnt;
             if (!ob) return;
             n_pair += 4 * __popc(ob);
-            if (open) sts_u32(q2_s + 4u * (n2 + __popc(ob & ((1u << lane) - 1u))), ((uint32_t)t << 7) | ((uint32_t)cl << 3) | (uint32_t)sidx);
+            if (open) sts_u32(q2_s + 4u * (n2 + __popc(ob & ((1u << lane) - 1u))), ((uint32_t)t << 8) | ((uint32_t)cl << 3) | (uint32_t)sidx);
             n2 += __popc(ob);
             __syncwarp();
             while (n2 >= 8) {
@@ -725,7 +730,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
         auto enqueue = [&](uint32_t todo, int cl) {
             if (todo == 0) return;
             if ((todo >> lane) & 1u)
-                sts_u32(q1_s + 4u * (n1 + __popc(todo & ((1u << lane) - 1u))), ((uint32_t)town << 4) | (uint32_t)cl);
+                sts_u32(q1_s + 4u * (n1 + __popc(todo & ((1u << lane) - 1u))), ((uint32_t)town << 5) | (uint32_t)cl);
             n1 += __popc(todo);
             __syncwarp();
             while (n1 >= 4) {
@@ -741,7 +746,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
             for (int k = 0; k < G::CW; k++) le[k] = p[k] - mn[k];  // guard <=> corner <= p
             return gather_mask<G::NG>(le);
         };
-        const int nch_tile = (int)min((int64_t)kWarps, nchunks - tile * kWarps);
+        const int nch_tile = (int)min((int64_t)NW, nchunks - tile * NW);
         const bool mine = (valid >> lane) & 1u;
         int cl = wsub;
         for (; cl + wpg < nch_tile; cl += 2 * wpg) {
@@ -777,39 +782,39 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 1) k3_owner_kernel(
             atomicAdd(&counters[6], n_exp);
         }
     }
-    consumer_sync(kWarps * 32);
-    write_rows<D, MODE>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids, zm);
+    consumer_sync(NW * 32);
+    write_rows<D, MODE, NW>(state, j0, nt, warp, lane, max_level, rows32, tie32, ext_rows32, host_mem, ext_ids, zm);
 }
 
-template <int D, int MODE>
+template <int D, int MODE, int NW>
 size_t owner_smem_bytes(int ngrp) {
-    using C = GeoK3<D, MODE>;
+    using C = GeoO<D, MODE, NW>;
     const size_t tpc = (size_t)ngrp * 32;
-    return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + C::PS + 1) + kWarps * C::QW);
+    return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + C::PS + 1) + NW * C::QW);
 }
 
-// Largest power-of-two task-group count (<= 16) whose state fits in shared memory; 0 if not even one.
-template <int D, int MODE>
-int owner_max_groups() {
-    int g = 16;
-    while (g >= 1 && owner_smem_bytes<D, MODE>(g) > (size_t)kSmemBytes) g >>= 1;
-    return g;
+// Largest task-group count dividing NW (every group gets NW / ngrp warps) whose state fits in shared memory and
+// that does not exceed `want`; 0 if not even one group fits.
+template <int D, int MODE, int NW>
+int owner_groups(int64_t want) {
+    int best = 0;
+    for (int g = 1; g <= NW; g++)
+        if (NW % g == 0 && owner_smem_bytes<D, MODE, NW>(g) <= (size_t)kSmemBytes && (g == 1 || g <= want)) best = g;
+    return best;
 }
 
-template <int D, int MODE>
+template <int D, int MODE, int NW>
 bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
                   cudaStream_t st) {
-    const int gmax = owner_max_groups<D, MODE>();
-    if (gmax < 1) return false;
     const int64_t range = j_end - j_begin;
     // groups per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t want = std::max<int64_t>(1, ceil_div(ceil_div(range, c.num_sms), 32));
-    int ngrp = 1;
-    while (ngrp * 2 <= gmax && ngrp * 2 <= want) ngrp *= 2;
-    const size_t smem = owner_smem_bytes<D, MODE>(ngrp);
-    SKY_CUDA(cudaFuncSetAttribute(k3_owner_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const int ngrp = owner_groups<D, MODE, NW>(want);
+    if (ngrp < 1) return false;
+    const size_t smem = owner_smem_bytes<D, MODE, NW>(ngrp);
+    SKY_CUDA(cudaFuncSetAttribute(k3_owner_kernel<D, MODE, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const unsigned blocks = (unsigned)ceil_div(range, ngrp * 32);
-    k3_owner_kernel<D, MODE><<<blocks, (kWarps + 1) * 32, smem, st>>>(
+    k3_owner_kernel<D, MODE, NW><<<blocks, (NW + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
         c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32, c.tie.as<uint32_t>(), ext_rows32,
@@ -863,7 +868,15 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
     const int design = tuning().k3_design;
     const bool want_o = design ? design == 'O' : MODE == kModeDims;
-    if (want_o && launch_owner<D, MODE>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
+    if (want_o) {
+        // design O with 24 warps (the group count divides 24: e.g. 3 groups of 8 warps at d = 10, where 16 warps
+        // fit only 2 groups): C5 K3 26.8 -> 20.2 ms, C2 0.5 -> 0.3 ms (profiles/r02_k3_warps_ab.md);
+        // k3_warps = 16 forces the 16-warp kernel
+        if constexpr (D <= 12)
+            if (tuning().k3_warps != 16 && launch_owner<D, MODE, 24>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st))
+                return;
+        if (launch_owner<D, MODE, kWarps>(c, j_begin, j_end, rows32, ext_rows32, host_mem, st)) return;
+    }
     // design A: one chunk per consumer warp per tile.  At d = 12, 24 consumer warps (70 registers, 2 ring stages
     // of 24 chunks) instead of 16 (89 registers, 4 stages of 16): more warps per SM sub-partition against K3's
     // fixed-latency ("wait") stalls.  With the round-2 expansion walk it measured H 94.2 -> 89.5 ms, C3A 39.3 ->
