@@ -864,10 +864,11 @@ void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
 template <int D, int MODE>
 void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t *ext_rows32, uint32_t *host_mem,
               cudaStream_t st) {
-    // Design O where its state fits and measured faster (the per-dimension tie-exact state: C5 34.3 -> 29.6
-    // ms); design A otherwise (H: A 92.8 ms vs O 97.5 ms).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
+    // Design O (task-owner warps) at d <= 12, where 24 warps fit 8 groups of tasks: H K3 86.7 (A, 24 warps) ->
+    // 83.4 ms, C3I 7.2 -> 6.2, C3A 33.9 -> 34.3, C5 (tie-exact state) 20.1 (round 1 with 16 warps: A 92.8 vs O
+    // 97.5 at H); design A above d = 12.  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
     const int design = tuning().k3_design;
-    const bool want_o = design ? design == 'O' : MODE == kModeDims;
+    const bool want_o = design ? design == 'O' : (MODE == kModeDims || D <= 12);
     if (want_o) {
         // design O with 24 warps (the group count divides 24: e.g. 3 groups of 8 warps at d = 10, where 16 warps
         // fit only 2 groups): C5 K3 26.8 -> 20.2 ms, C2 0.5 -> 0.3 ms (profiles/r02_k3_warps_ab.md);
