@@ -17,9 +17,9 @@ Nothing here comes from the CUDA path.  The GPU test ``tests/test_gpu_digest.py`
 output built through the bench launch path and compares it with these values.
 
 The run is chunked and resumable (Oracle B on H takes about 2 h on 8 cores): every chunk of
-``CHUNK`` points is stored under ``.oracle_work/<cfg>/`` (git- and gpurun-ignored) and skipped when
-present.  The wall and CPU time of every chunk is recorded, so the file also holds a full-size,
-un-extrapolated Oracle B timing on this host.
+``CHUNK`` points is stored under ``.oracle_work/<cfg>/`` (git-ignored; ``SKYCUBE_ORACLE_WORK`` moves it, e.g.
+out of the tree for C4's 8 GB of rows) and skipped when present.  The wall and CPU time of every chunk is
+recorded, so the file also holds a full-size, un-extrapolated Oracle B timing on this host.
 
 Usage: ``OMP_NUM_THREADS=8 nice -n 19 python tools/oracle_digest.py H C3A C5 [C4]``
 """
@@ -43,13 +43,14 @@ import datagen  # noqa: E402
 import oracle   # noqa: E402
 
 GOLDEN = os.path.join(ROOT, "tests", "golden", "fullsize_digests.json")
-WORK = os.path.join(ROOT, ".oracle_work")
+WORK = os.environ.get("SKYCUBE_ORACLE_WORK") or os.path.join(ROOT, ".oracle_work")
 CHUNK = 8192
 BLOCK = 4096
 
 
 def sha(a: np.ndarray) -> str:
-    return hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+    # hashes the array's buffer in place (C4's 28 GB lattice must not be copied)
+    return hashlib.sha256(memoryview(np.ascontiguousarray(a)).cast("B")).hexdigest()
 
 
 def file_sha(path: str) -> str:
