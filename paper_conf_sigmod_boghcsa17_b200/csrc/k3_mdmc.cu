@@ -113,6 +113,13 @@ __device__ __forceinline__ uint32_t gather_mask(const uint32_t *v) {
 }
 
 // Bits delta_low (0..31) that are subsets of x (x < 32): the word pattern of sub(x) in the low 5 dims.
+// the same as a table (warp-uniform index: one constant-cache load instead of ~10 instructions)
+__constant__ uint32_t kSub5[32] = {
+    0x00000001u, 0x00000003u, 0x00000005u, 0x0000000fu, 0x00000011u, 0x00000033u, 0x00000055u, 0x000000ffu,
+    0x00000101u, 0x00000303u, 0x00000505u, 0x00000f0fu, 0x00001111u, 0x00003333u, 0x00005555u, 0x0000ffffu,
+    0x00010001u, 0x00030003u, 0x00050005u, 0x000f000fu, 0x00110011u, 0x00330033u, 0x00550055u, 0x00ff00ffu,
+    0x01010101u, 0x03030303u, 0x05050505u, 0x0f0f0f0fu, 0x11111111u, 0x33333333u, 0x55555555u, 0xffffffffu};
+
 __device__ __forceinline__ uint32_t sub5(uint32_t x) {
     uint32_t t = 1u;
     if (x & 1u) t |= t << 1;
@@ -233,7 +240,7 @@ __device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t 
                                        int lane) {
     using G = Geo<D>;
     constexpr int WB = G::WB;
-    const uint32_t lh = L >> 5, lb = sub5(L & 31u);
+    const uint32_t lh = L >> 5, lb = kSub5[L & 31u];
     if (MODE == kModeDims) {
         bool changed = false;  // warp-uniform
         for (uint32_t s = S; s; s &= s - 1) {  // D_i |= sub(L) for every i in S
@@ -256,12 +263,12 @@ __device__ __forceinline__ void expand(uint32_t st_s, uint32_t *tie_g, uint32_t 
     }
     // B_{p notin S+} |= sub(S) (strict dominance propagates), unless already there
     if (!((lds_u32(st_s + 4u * (S >> 5)) >> (S & 31)) & 1u)) {
-        const uint32_t sb = sub5(S & 31u);
+        const uint32_t sb = kSub5[S & 31u];
         coop_words<WB>(S >> 5, lane, [&](uint32_t w) { red_or_s(st_s + 4u * w, sb); });
     }
     if (L == S) return;
     // ties: B_{p notin S} |= sub(L) \ sub(E), E = B_{q=p}  (reading Q3)
-    const uint32_t E = L & ~S, eh = E >> 5, eb = sub5(E & 31u);
+    const uint32_t E = L & ~S, eh = E >> 5, eb = kSub5[E & 31u];
     if (MODE == kModeGlobalTie) tie_row_mark(tflag_s, lane);
     coop_words<WB>(lh, lane, [&](uint32_t w) {
         const uint32_t bits = (w & ~eh) ? lb : (lb & ~eb);
@@ -657,9 +664,13 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     load_row_s<G::CW>(pV_s + 4u * (town * CWV), p);
     const uint32_t st_own = st_s + 4u * (town * C::PS);
     unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
+    // ring barriers as 32-bit shared addresses kept in registers, position (stage, phase) kept incrementally
+    // (a generic->shared conversion per wait/arrival was ~4% of this kernel's instructions at H, ncu r02)
+    const uint32_t full_s = smem_addr(bars), empty_s = full_s + 8u * kStages;
+    uint32_t stage = 0, phase = 0;
     for (int64_t tile = 0; tile < ntiles; tile++) {
-        ring.wait(tile);
-        const uint32_t stg_s = ring_s + 4u * (uint32_t)(tile % kStages) * (uint32_t)C::TW;
+        mbar_wait_s(full_s + 8u * stage, phase);
+        const uint32_t stg_s = ring_s + 4u * stage * (uint32_t)C::TW;
 
         // pair pass over 8 queued (task, chunk, sub-chunk) items: lane (k, r) = item k, member r
         auto pair_pass = [&](int base, int cnt) {
@@ -770,7 +781,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
         // every read of the stage has completed (values consumed) before it is handed back to the producer
         __threadfence_block();
         __syncwarp();
-        if (lane == 0) ring.release(tile);
+        if (lane == 0) mbar_arrive_s(empty_s + 8u * stage);
+        if (++stage == (uint32_t)kStages) {
+            stage = 0;
+            phase ^= 1u;
+        }
     }
     if (counters) {
         for (int o = 16; o; o >>= 1) n_miss += __shfl_xor_sync(0xffffffffu, n_miss, o);

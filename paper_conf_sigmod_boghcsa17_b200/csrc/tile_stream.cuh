@@ -60,6 +60,21 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) 
     } while (!done);
 }
 
+// 32-bit shared-window forms for kernels that keep barrier addresses in registers (design O of K3).
+__device__ __forceinline__ void mbar_wait_s(uint32_t addr, uint32_t parity) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(done)
+            : "r"(addr), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void mbar_arrive_s(uint32_t addr) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(addr) : "memory");
+}
+
 // Double-buffered stream of fixed-size tiles (bytes multiple of 16, 16-B aligned source).
 struct TileStream2 {
     uint64_t *bar;  // [2] in shared memory
