@@ -18,7 +18,7 @@ SKYCUBE_K3_WARPS=24 timeout 600 python bench.py --cpu-seconds 2 --no-e2e 2>/dev/
 timeout 900 python bench.py --impl reference --steps 2 --warmup 1 2>/dev/null | tail -1 > gpurun_out/ev_bench_H_reference.json
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_launches_H.csv \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > gpurun_out/ev_ncu_launch.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k3_mdmc -c 1 -f -o gpurun_out/ev_prof_k3_mdmc_H \
-  python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k3_mdmc_H.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k3_ -c 1 -f -o gpurun_out/ev_prof_k3_H \
+  python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k3_H.log 2>&1
 cat gpurun_out/ev_tests.log gpurun_out/ev_smoke.log
 for f in gpurun_out/ev_bench_*.json; do echo "$f: $(head -c 160 $f)"; done

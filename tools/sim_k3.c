@@ -12,7 +12,7 @@
  *              holds M_g skips without its own mask; a warp-iteration is free iff all 32 lanes skip
  *   gtile      per (group, tile of 16 chunks): same with the tile's lower corner
  * Usage: sim_k3 points.f32 n d ngroups_sample task_order(0=id,1=morton) chunk_order(0=sum,1=morton,2=coarse)
- *        [chunk_size=32] [sub_size=4]
+ *        [chunk_size=32] [sub_size=4] [box_shift=0] [sub_shift=0]
  */
 #include <stdint.h>
 #include <stdio.h>
@@ -66,6 +66,7 @@ int main(int argc, char **argv) {
     const int nsample = atoi(argv[4]), task_order = atoi(argv[5]), chunk_order = atoi(argv[6]);
     const int CS = argc > 7 ? atoi(argv[7]) : 32, SS = argc > 8 ? atoi(argv[8]) : 4, NSUB = CS / SS;
     const int BOXSHIFT = argc > 9 ? atoi(argv[9]) : 0;  /* box test on codes >> BOXSHIFT (coarser, still sound) */
+    const int SUBSHIFT = argc > 10 ? atoi(argv[10]) : 0;  /* sub-corner test on codes >> SUBSHIFT */
     float *X = malloc(sizeof(float) * N * D);
     FILE *f = fopen(argv[1], "rb");
     if (fread(X, sizeof(float), (size_t)N * D, f) != (size_t)N * D) return 2;
@@ -270,7 +271,12 @@ int main(int argc, char **argv) {
                     }
                     for (int s = 0; s < NSUB; s++) {
                         n_sub++;
-                        if (bit(sp, le_mask(sub + ((long)c * NSUB + s) * D, pc))) continue;
+                        {
+                            const uint16_t *sc = sub + ((long)c * NSUB + s) * D;
+                            uint32_t Ms = 0;
+                            for (int i = 0; i < D; i++) Ms |= (uint32_t)((sc[i] >> SUBSHIFT) <= (pc[i] >> SUBSHIFT)) << i;
+                            if (bit(sp, Ms)) continue;
+                        }
                         for (int r = 0; r < SS; r++) {
                             const int kq = c * CS + s * SS + r;
                             if (kq >= m) continue;
