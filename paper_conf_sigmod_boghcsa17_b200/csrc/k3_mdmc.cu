@@ -601,7 +601,7 @@ template <int D, int MODE, int NW>
 __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
-    int64_t j_end, uint32_t inexact, int ngrp, int max_level, uint32_t *__restrict__ rows32,
+    int64_t j_end, uint32_t inexact, int ngrp, int tpc, int max_level, uint32_t *__restrict__ rows32,
     uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters,
     uint32_t *__restrict__ host_mem, const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
@@ -611,7 +611,8 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     constexpr int kStages = C::kStages;
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
-    const int tpc = ngrp * 32;
+    // tpc = ngrp * 32, or fewer than 32 tasks in one partial group when the 2^d-bit state of 32 tasks does not
+    // fit (d >= 15); lanes past tpc then address task tpc - 1 and own nothing
     uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits
     uint32_t *state = pV + tpc * CWV;          // [tpc][PS]
     uint32_t *zm = state + tpc * C::PS;        // [tpc] Z_p (kModeDims)
@@ -660,9 +661,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     const int wpg = NW / ngrp, grp = warp / wpg, wsub = warp % wpg;
     const int town = grp * 32 + lane;                         // this lane's task
     const uint32_t valid = __ballot_sync(0xffffffffu, town < nt);
+    const uint32_t st_own = st_s + 4u * (min(town, tpc - 1) * C::PS);
     uint32_t p[G::CW];
-    load_row_s<G::CW>(pV_s + 4u * (town * CWV), p);
-    const uint32_t st_own = st_s + 4u * (town * C::PS);
+    load_row_s<G::CW>(pV_s + 4u * (min(town, tpc - 1) * CWV), p);
     unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     // ring barriers as 32-bit shared addresses kept in registers, position (stage, phase) kept incrementally
     // (a generic->shared conversion per wait/arrival was ~4% of this kernel's instructions at H, ncu r02)
@@ -802,9 +803,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
 }
 
 template <int D, int MODE, int NW>
-size_t owner_smem_bytes(int ngrp) {
+size_t owner_smem_bytes(int tasks) {
     using C = GeoO<D, MODE, NW>;
-    const size_t tpc = (size_t)ngrp * 32;
+    const size_t tpc = (size_t)tasks;
     return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + C::PS + 1) + NW * C::QW);
 }
 
@@ -814,7 +815,7 @@ template <int D, int MODE, int NW>
 int owner_groups(int64_t want) {
     int best = 0;
     for (int g = 1; g <= NW; g++)
-        if (NW % g == 0 && owner_smem_bytes<D, MODE, NW>(g) <= (size_t)kSmemBytes && (g == 1 || g <= want)) best = g;
+        if (NW % g == 0 && owner_smem_bytes<D, MODE, NW>(g * 32) <= (size_t)kSmemBytes && (g == 1 || g <= want)) best = g;
     return best;
 }
 
@@ -824,14 +825,21 @@ bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint
     const int64_t range = j_end - j_begin;
     // groups per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t want = std::max<int64_t>(1, ceil_div(ceil_div(range, c.num_sms), 32));
-    const int ngrp = owner_groups<D, MODE, NW>(want);
-    if (ngrp < 1) return false;
-    const size_t smem = owner_smem_bytes<D, MODE, NW>(ngrp);
+    int ngrp = owner_groups<D, MODE, NW>(want), tpc = ngrp * 32;
+    if (ngrp < 1) {
+        // one partial group: as many tasks as the shared memory holds (d = 16: 22 tasks of 8 KB state)
+        ngrp = 1;
+        tpc = 0;
+        while (tpc < 31 && owner_smem_bytes<D, MODE, NW>(tpc + 1) <= (size_t)kSmemBytes) tpc++;
+        if (tpc < 1) return false;
+        tpc = (int)std::min<int64_t>(tpc, std::max<int64_t>(1, ceil_div(range, c.num_sms)));
+    }
+    const size_t smem = owner_smem_bytes<D, MODE, NW>(tpc);
     SKY_CUDA(cudaFuncSetAttribute(k3_owner_kernel<D, MODE, NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    const unsigned blocks = (unsigned)ceil_div(range, ngrp * 32);
+    const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_owner_kernel<D, MODE, NW><<<blocks, (NW + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp,
+        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp, tpc,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32, c.tie.as<uint32_t>(), ext_rows32,
         c.counters.as<unsigned long long>(), host_mem, c.ext_ids.as<int32_t>());
     c.L.count++;
@@ -881,9 +889,12 @@ void launch_t(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
               cudaStream_t st) {
     // Design O (task-owner warps) at d <= 12, where 24 warps fit 8 groups of tasks: H K3 86.7 (A, 24 warps) ->
     // 83.4 ms, C3I 7.2 -> 6.2, C3A 33.9 -> 34.3, C5 (tie-exact state) 20.1 (round 1 with 16 warps: A 92.8 vs O
-    // 97.5 at H); design A above d = 12.  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
+    // 97.5 at H); and at d = 16 with one partial group of 22 tasks (task codes in registers instead of reloaded
+    // per chunk, competitor rows read from the stage on demand): C4 K3 644 -> 615 ms.  Design A at d = 13..15,
+    // where both measured within 1% (A 300K: d = 13 31.8 / 31.6 ms, d = 14 45.3 / 45.0, d = 15 71.3 / 72.1;
+    // profiles/r02_k3_ab_s2.md).  skycube_set_tuning("k3_design", 'A' | 'O') forces one.
     const int design = tuning().k3_design;
-    const bool want_o = design ? design == 'O' : (MODE == kModeDims || D <= 12);
+    const bool want_o = design ? design == 'O' : (MODE == kModeDims || D <= 12 || D == 16);
     if (want_o) {
         // design O with 24 warps (the group count divides 24: e.g. 3 groups of 8 warps at d = 10, where 16 warps
         // fit only 2 groups): C5 K3 26.8 -> 20.2 ms, C2 0.5 -> 0.3 ms (profiles/r02_k3_warps_ab.md);

@@ -4,6 +4,8 @@ from __future__ import annotations
 import json
 import os
 
+import functools
+
 import numpy as np
 import pytest
 
@@ -240,6 +242,30 @@ def test_k3_designs_and_modes(tuning, design, mode, case):
     assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
     off, ids = oracle.lattice(want, d)
     assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)
+
+
+@pytest.mark.parametrize("design", ["A", "O"])
+@pytest.mark.parametrize("mode", ["0", "1"])
+@pytest.mark.parametrize("case", [("A", 3000, 16, 906), ("A", 2600, 15, 907), ("grid", 900, 16, 908)])
+def test_k3_designs_high_d(tuning, design, mode, case):
+    """d = 15 and 16, both designs: design O with one partial group (fewer than 32 tasks per CTA when 32 tasks'
+    2^d-bit state does not fit in shared memory; the lanes past the last task own nothing), several tiles with
+    ragged tails, both B_{p notin S+}-probe state modes; every row and the lattice must equal the oracle."""
+    tuning("k3_design", design)
+    tuning("k3_mode", int(mode))
+    x, want, off, ids = _high_d_case(*case)
+    r = sky.skycube_build(x)
+    bad = np.nonzero((r["rows"] != want).any(axis=1))[0]
+    assert bad.size == 0, f"{bad.size} rows differ, first {bad[:5]}"
+    assert np.array_equal(r["offsets"], off) and np.array_equal(r["ids"], ids)
+
+
+@functools.lru_cache(maxsize=None)
+def _high_d_case(dist, n, d, seed):
+    x = datagen.small_int_grid(n, d, 3, seed) if dist == "grid" else datagen.generate(dist, n, d, seed)
+    want = oracle.rows_b(x)
+    off, ids = oracle.lattice(want, d)
+    return x, want, off, ids
 
 
 @pytest.mark.parametrize("warps", [16, 24])

@@ -12,7 +12,7 @@
  *              holds M_g skips without its own mask; a warp-iteration is free iff all 32 lanes skip
  *   gtile      per (group, tile of 16 chunks): same with the tile's lower corner
  * Usage: sim_k3 points.f32 n d ngroups_sample task_order(0=id,1=morton) chunk_order(0=sum,1=morton,2=coarse)
- *        [chunk_size=32] [sub_size=4] [box_shift=0] [sub_shift=0]
+ *        [chunk_size=32] [sub_size=4] [box_shift=0] [sub_shift=0] [prelude=0]
  */
 #include <stdint.h>
 #include <stdio.h>
@@ -67,6 +67,9 @@ int main(int argc, char **argv) {
     const int CS = argc > 7 ? atoi(argv[7]) : 32, SS = argc > 8 ? atoi(argv[8]) : 4, NSUB = CS / SS;
     const int BOXSHIFT = argc > 9 ? atoi(argv[9]) : 0;  /* box test on codes >> BOXSHIFT (coarser, still sound) */
     const int SUBSHIFT = argc > 10 ? atoi(argv[10]) : 0;  /* sub-corner test on codes >> SUBSHIFT */
+    /* prelude: before the global order, each group visits the PRE static-tree (Morton) chunks on either side of
+     * its own position (meaningful with task_order = 1: group g = the members of chunk g) */
+    const int PRE = argc > 11 ? atoi(argv[11]) : 0;
     float *X = malloc(sizeof(float) * N * D);
     FILE *f = fopen(argv[1], "rb");
     if (fread(X, sizeof(float), (size_t)N * D, f) != (size_t)N * D) return 2;
@@ -230,15 +233,29 @@ int main(int argc, char **argv) {
                 if (c > U[i]) U[i] = c;
             }
         }
-        for (int t = 0; t < ntl; t++) {
-            /* tile-level group test */
-            const uint32_t Mt = le_mask(tcorner + (long)t * D, U);
-            int all = 1;
-            for (int l = 0; l < 32; l++) all &= bit(st + l * W, Mt);
-            t_iters++;
-            if (all) t_warp_free++;
-            for (int k = t * 16; k < nch && k < t * 16 + 16; k++) {
-                const int c = corder[k];
+        for (int t = -1; t < ntl; t++) {
+            int all = 0, k0, k1;
+            if (t < 0) { /* prelude */
+                k0 = -2 * PRE - 1;
+                k1 = PRE > 0 ? 0 : k0;
+            } else {
+                /* tile-level group test */
+                const uint32_t Mt = le_mask(tcorner + (long)t * D, U);
+                all = 1;
+                for (int l = 0; l < 32; l++) all &= bit(st + l * W, Mt);
+                t_iters++;
+                if (all) t_warp_free++;
+                k0 = t * 16;
+                k1 = k0 + 16 < nch ? k0 + 16 : nch;
+            }
+            for (int k = k0; k < k1; k++) {
+                int c;
+                if (k < 0) {
+                    c = g + (k + PRE + 1);
+                    if (c < 0 || c >= nch) continue;
+                } else {
+                    c = corder[k];
+                }
                 const uint16_t *cc = corner + (long)c * D;
                 const uint32_t Mg = le_mask(cc, U);
                 int allg = 1;
