@@ -58,6 +58,7 @@ struct Ctx {
     uint32_t W = 1;
     uint32_t exact_mask = 0;    // bit i <=> the codes of dimension i are injective (dense ranks)
     uint32_t R[kMaxD] = {0};    // distinct values per dimension
+    uint64_t cshift = 0;        // coarse-code shift of dimension i in bits 4i..4i+3 (K3 corner tests)
     int64_t m = 0;              // |S+(P)|
     int max_level = 0;          // partial skycube (Appendix A.2): report only |delta| <= max_level (0 = d)
     bool prepared = false, ext_ready = false;
@@ -85,7 +86,7 @@ struct Ctx {
     DevBuf q_ord;       // u32 [m*d]
     DevBuf tie;         // u32 tiled rows: tie contributions to B_{p notin S}
     DevBuf chunks_all;  // u32 [n/32][kRecAll][cw]  chunk records of all points (K1 competitors)
-    DevBuf chunks_ext;  // u32 [m/32][kRecExt][cw]  chunk records of S+ with sub-chunk corners (K3 competitors)
+    DevBuf chunks_ext;  // u32 [m/32][rec_ext_words(cw)]  chunk records of S+ with coarse corners (K3 competitors)
     DevBuf chunk_keys, chunk_perm, q_codes_alt, q_ord_alt;  // chunk visiting order (strongest corner first)
     DevBuf supers_all;  // u32 [tiles][super_words(cw)]  lower corner of each tile of 16 chunks (K1)
     int64_t nchunks_all = 0, nchunks_ext = 0;
@@ -138,7 +139,15 @@ constexpr int64_t kChunkTilePad = 512;  // extra never-better points so chunk ti
 constexpr int kTileChunks = 16;         // chunks per competitor tile (one super-chunk of 512 points)
 constexpr int kSubSize = 4;             // points per sub-chunk (K3 level below the chunk)
 constexpr int kRecAll = 33;             // K1 chunk record rows: 32 points + corner
-constexpr int kRecExt = 33 + 32 / kSubSize;  // K3 chunk record rows: + 8 sub-chunk corners
+// K3 chunk records: the 32 members' 15-bit code words (cw words each, the pair pass), then the chunk's lower
+// corner and the lower corners of its 8 sub-chunks as COARSE codes: 7 bits per dimension, four dimensions per
+// 32-bit word (kCoarseWords words per row, d <= 16), for the corner tests (box and sub-chunk passes).  The
+// coarse code of dimension i is min(code >> cshift_i, 127), cshift_i the smallest shift that maps the
+// dimension's codes into 7 bits (0 when it has <= 128 distinct values): monotone, so a coarse lower corner
+// below p in dimension i is implied by the fine one and every corner test stays sound (Λ3, Λ4).
+constexpr int kCoarseWords = 4;
+constexpr int kCoarseRows = 1 + 32 / kSubSize;  // chunk corner + 8 sub-chunk corners
+__host__ __device__ inline int rec_ext_words(int cw) { return 32 * cw + kCoarseRows * kCoarseWords; }
 inline int super_words(int cw) { return (cw + 3) & ~3; }  // super-corner record words (16-byte multiple)
 
 }  // namespace sky

@@ -84,14 +84,14 @@ template <int D, int MODE, int NW = kWarps, int ST = 0>
 struct GeoK3 {
     static constexpr int PER = (MODE == kModeGlobalTie ? 1 : MODE == kModeSmemTie ? 2 : D + 1) * Geo<D>::WB;
     static constexpr int PS = PER | 1;                                   // odd task stride (bank spread)
-    static constexpr int CWP = Geo<D>::CW | 1;                           // odd code stride (box pass)
     static constexpr int CWV = (Geo<D>::CW + 3) & ~3;                    // 16-byte code stride (pair pass)
-    static constexpr int REC = kRecExt * Geo<D>::CW;                     // chunk record words
+    static constexpr int REC = 32 * Geo<D>::CW + kCoarseRows * kCoarseWords;  // chunk record words (ctx.cuh)
+    static constexpr int CO = 32 * Geo<D>::CW;                           // coarse chunk corner; sub-corner s at CO+4+4s
     static constexpr int TW = NW * REC;                                  // tile words (one chunk per consumer warp)
     static constexpr int kStages = ST > 0 ? ST : NW > kWarps && D < 15 ? SKY_K3_STAGES_WIDE : k3_stages<D>();
     static constexpr int RING = 4 * kStages + kStages * TW;              // barriers + stages (words)
     static constexpr int QW = 96;                                        // per-warp queue words (tasks, items)
-    static constexpr int ROW = PS + CWP + CWV + 1;                       // words per task (+ Z_p)
+    static constexpr int ROW = PS + kCoarseWords + CWV + 1;              // words per task: state, coarse, fine, Z_p
     static constexpr int NT0 = (kSmemBytes / 4 - RING - NW * QW - 64) / ROW;
     static constexpr int NT = NT0 < 1024 ? NT0 : 1024;                   // tasks per CTA
     static size_t smem_bytes(int tpc) { return sizeof(uint32_t) * ((size_t)RING + (size_t)tpc * ROW + NW * QW); }
@@ -110,6 +110,35 @@ __device__ __forceinline__ uint32_t gather_mask(const uint32_t *v) {
         m = __funnelshift_l(y, m, 4);       // (m << 4) | (y >> 28)
     }
     return m;
+}
+
+// Coarse corner test (chunk records, ctx.cuh): 7-bit codes, four dimensions per word (byte k = dimension 4g+k),
+// the task side carrying a guard bit per byte: x = (p | 0x80808080) - corner has the guard bit of byte k set
+// <=> corner_k <= p_k (no borrow crosses a byte).  Word g -> mask bits 4g..4g+3 by the same carry-free multiply.
+template <int NQ>
+__device__ __forceinline__ uint32_t gather_coarse(const uint32_t *x) {
+    uint32_t m = 0;
+#pragma unroll
+    for (int g = NQ - 1; g >= 0; g--) m = __funnelshift_l((x[g] & 0x80808080u) * 0x00204081u, m, 4);
+    return m;
+}
+
+// The coarse code row of task t (four words, guard bits set) from its fine 15-bit code words; dimensions >= D are 0.
+template <int D, int CW>
+__device__ __forceinline__ void coarse_row(const uint32_t *fine, uint64_t cshift, uint32_t *out) {
+#pragma unroll
+    for (int g = 0; g < kCoarseWords; g++) {
+        uint32_t w = 0x80808080u;
+#pragma unroll
+        for (int b = 0; b < 4; b++) {
+            const int i = 4 * g + b;
+            if (i < D) {
+                const uint32_t code = (fine[i >> 1] >> (16 * (i & 1))) & 0x7fffu;
+                w |= min(code >> ((cshift >> (4 * i)) & 15u), 127u) << (8 * b);
+            }
+        }
+        out[g] = w;
+    }
 }
 
 // Bits delta_low (0..31) that are subsets of x (x < 32): the word pattern of sub(x) in the low 5 dims.
@@ -366,24 +395,25 @@ template <int D, int MODE, int NW>
 __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
-    int64_t j_end, uint32_t inexact, int tpc, int max_level, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
+    int64_t j_end, uint32_t inexact, uint64_t cshift, int tpc, int max_level, uint32_t *__restrict__ rows32, uint32_t *__restrict__ tie32,
     uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters, uint32_t *__restrict__ host_mem,
     const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoK3<D, MODE, NW>;
-    constexpr int CWP = C::CWP, CWV = C::CWV, REC = C::REC;
+    constexpr int CWV = C::CWV, REC = C::REC, NQ = (D + 3) / 4;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     constexpr int kStages = C::kStages;
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
-    uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits (broadcast rows)
-    uint32_t *pH = pV + tpc * CWV;             // [tpc][CWP] the same, odd stride (per-lane rows)
-    uint32_t *state = pH + tpc * CWP;          // [tpc][PS]
+    uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits (pair pass)
+    uint32_t *pC = pV + tpc * CWV;             // [tpc][4] coarse task codes with guard bits (corner tests)
+    uint32_t *state = pC + tpc * kCoarseWords; // [tpc][PS]
     uint32_t *zm = state + tpc * C::PS;        // [tpc] Z_p (kModeDims)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint32_t *wq = zm + tpc + warp * C::QW;    // per-warp queue of opened tasks (<= 3 + 32 entries)
     uint32_t *iq = wq + 40;                    // per-warp queue of opened (task, sub-chunk) items (<= 7 + 32)
     const uint32_t st_s = smem_addr(state), wq_s = smem_addr(wq), iq_s = smem_addr(iq), pV_s = smem_addr(pV);
+    const uint32_t pC_s = smem_addr(pC);
     const uint32_t zm_s = smem_addr(zm);  // kModeGlobalTie: per-task tie-row flags (kModeDims: Z_p)
     const int64_t j0 = j_begin + (int64_t)blockIdx.x * tpc;
     const int nt = (int)min((int64_t)tpc, j_end - j0);
@@ -395,9 +425,10 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
         uint32_t w = t < nt ? p_codes[(j0 + t) * G::CW + k] : 0u;
         if (2 * k >= D) w &= 0xffff0000u;  // padding dimensions: p = 0 never passes q <= p (q pad = 1)
         if (2 * k + 1 >= D) w &= 0x0000ffffu;
-        pH[t * CWP + k] = w | kGuard;
         pV[t * CWV + k] = w | kGuard;
     }
+    __syncthreads();
+    for (int t = threadIdx.x; t < tpc; t += blockDim.x) coarse_row<D, G::CW>(pV + t * CWV, cshift, pC + t * kCoarseWords);
     if (MODE == kModeDims) {
         // Z_p = { i : p[i] is the minimum of dimension i } (exact keys); K starts as sub(Z_p)
         for (int t = threadIdx.x; t < tpc; t += blockDim.x) {
@@ -428,15 +459,13 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
     for (int64_t tile = 0; tile < ntiles; tile++) {
         ring.wait(tile);
         const uint32_t *rec = ring.stage(tile) + warp * REC;
-        // this lane's competitor, the chunk corner, and the corner of sub-chunk (lane & 7) — the level below
-        // the chunk in the static tree (4 points) — all read before the stage is released
-        uint32_t q[G::CW], mn[G::CW], sc[G::CW];
+        // this lane's competitor, the chunk's coarse corner, and the coarse corner of sub-chunk (lane & 7) — the
+        // level below the chunk in the static tree (4 points) — all read before the stage is released
+        uint32_t q[G::CW], mn[kCoarseWords], sc[kCoarseWords];
 #pragma unroll
-        for (int k = 0; k < G::CW; k++) {
-            q[k] = rec[lane * G::CW + k];
-            mn[k] = rec[32 * G::CW + k];
-            sc[k] = rec[(33 + (lane & 7)) * G::CW + k];
-        }
+        for (int k = 0; k < G::CW; k++) q[k] = rec[lane * G::CW + k];
+        load_row<kCoarseWords>(rec + C::CO, mn);
+        load_row<kCoarseWords>(rec + C::CO + kCoarseWords * (1 + (lane & 7)), sc);
         // The loads above are still in flight (their values are first used much later): complete them before
         // the stage is handed back to the TMA producer, or the next tile's bulk copy can overwrite the stage
         // under them (observed as rare missing dominations at d >= 13 without this fence).
@@ -465,7 +494,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
             uint32_t L = 0, S = 0;
             if (miss) {
                 n_miss++;
-                exact_masks<D>(pH + t * CWP, qq, M, inexact, q_ord + (c * 32 + src) * D, p_ord + (j0 + t) * D, L, S);
+                exact_masks<D>(pV + t * CWV, qq, M, inexact, q_ord + (c * 32 + src) * D, p_ord + (j0 + t) * D, L, S);
                 if (S != 0 && L != M && ((lds_u32(st_s + 4u * (uint32_t)(t * C::PS + (L >> 5))) >> (L & 31)) & 1u))
                     S = 0;  // exact L covered
             }
@@ -489,11 +518,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
         auto sub_pass = [&](int base, int cnt) {
             const int u = lane >> 3;
             const int t = (int)lds_u32(wq_s + 4u * (base + min(u, cnt - 1)));
-            uint32_t x[G::CW];
-            load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
+            uint32_t x[kCoarseWords];
+            load_row_s<kCoarseWords>(pC_s + 4u * (t * kCoarseWords), x);
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) x[k] -= sc[k];  // guard <=> sub-corner <= p
-            const uint32_t Ms = gather_mask<G::NG>(x);
+            for (int k = 0; k < NQ; k++) x[k] -= sc[k];  // guard <=> coarse sub-corner <= p
+            const uint32_t Ms = gather_coarse<NQ>(x);
             const uint32_t ws = lds_u32(st_s + 4u * (t * C::PS + (Ms >> 5)));
             const bool open = u < cnt && !(__funnelshift_r(ws, ws, Ms) & 1u);
             const uint32_t ob = __ballot_sync(0xffffffffu, open);
@@ -525,12 +554,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_mdmc_kernel(
             __syncwarp();
         };
         auto box_test = [&](int tt, uint32_t &Mb) {
-            uint32_t le[G::CW];
-            // scalar loads from the odd-stride row copy: conflict-free across the 32 task lanes (two LDS.128
-            // from the 16-byte-stride copy measured 5% slower at H: 4+ wavefronts each, longer latency)
+            uint32_t le[kCoarseWords];
+            load_row_s<kCoarseWords>(pC_s + 4u * (tt * kCoarseWords), le);  // one LDS.128: 4 conflict-free phases
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) le[k] = pH[tt * CWP + k] - mn[k];  // guard <=> corner <= p
-            Mb = gather_mask<G::NG>(le);
+            for (int k = 0; k < NQ; k++) le[k] -= mn[k];  // guard <=> coarse corner <= p
+            Mb = gather_coarse<NQ>(le);
         };
         int g = 0;
         for (; g + 1 < ngroups; g += 2) {
@@ -601,20 +629,21 @@ template <int D, int MODE, int NW>
 __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     const uint32_t *__restrict__ p_codes, const uint32_t *__restrict__ p_ord, const uint32_t *__restrict__ chunks,
     const uint32_t *__restrict__ q_ord, const uint32_t *__restrict__ minord, int64_t nchunks, int64_t j_begin,
-    int64_t j_end, uint32_t inexact, int ngrp, int tpc, int max_level, uint32_t *__restrict__ rows32,
+    int64_t j_end, uint32_t inexact, uint64_t cshift, int ngrp, int tpc, int max_level, uint32_t *__restrict__ rows32,
     uint32_t *__restrict__ tie32, uint32_t *__restrict__ ext_rows32, unsigned long long *__restrict__ counters,
     uint32_t *__restrict__ host_mem, const int32_t *__restrict__ ext_ids) {
     using G = Geo<D>;
     using C = GeoO<D, MODE, NW>;
-    constexpr int CWV = C::CWV, REC = C::REC;
+    constexpr int CWV = C::CWV, REC = C::REC, NQ = (D + 3) / 4;
     extern __shared__ __align__(128) uint32_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);
     constexpr int kStages = C::kStages;
     const TileRing<kStages> ring{bars, bars + kStages, smem + 4 * kStages, (uint32_t)C::TW};
     // tpc = ngrp * 32, or fewer than 32 tasks in one partial group when the 2^d-bit state of 32 tasks does not
     // fit (d >= 15); lanes past tpc then address task tpc - 1 and own nothing
-    uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits
-    uint32_t *state = pV + tpc * CWV;          // [tpc][PS]
+    uint32_t *pV = smem + C::RING;             // [tpc][CWV] task codes with guard bits (pair pass)
+    uint32_t *pC = pV + tpc * CWV;             // [tpc][4] coarse task codes with guard bits (corner tests)
+    uint32_t *state = pC + tpc * kCoarseWords; // [tpc][PS]
     uint32_t *zm = state + tpc * C::PS;        // [tpc] Z_p (kModeDims)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint32_t *q1 = zm + tpc + warp * C::QW;    // opened (task, chunk) items (<= 3 + 32)
@@ -631,6 +660,8 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
         if (2 * k + 1 >= D) w &= 0x0000ffffu;
         pV[t * CWV + k] = w | kGuard;
     }
+    __syncthreads();
+    for (int t = threadIdx.x; t < tpc; t += blockDim.x) coarse_row<D, G::CW>(pV + t * CWV, cshift, pC + t * kCoarseWords);
     if (MODE == kModeDims) {
         for (int t = threadIdx.x; t < tpc; t += blockDim.x) {
             uint32_t z = 0;
@@ -662,8 +693,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
     const int town = grp * 32 + lane;                         // this lane's task
     const uint32_t valid = __ballot_sync(0xffffffffu, town < nt);
     const uint32_t st_own = st_s + 4u * (min(town, tpc - 1) * C::PS);
-    uint32_t p[G::CW];
-    load_row_s<G::CW>(pV_s + 4u * (min(town, tpc - 1) * CWV), p);
+    uint32_t p[kCoarseWords];  // this lane's coarse task codes (corner tests)
+    load_row_s<kCoarseWords>(smem_addr(pC) + 4u * (min(town, tpc - 1) * kCoarseWords), p);
+    const uint32_t pC_s = smem_addr(pC);
     unsigned long long n_box = 0, n_sub = 0, n_pair = 0, n_miss = 0, n_exp = 0;
     // ring barriers as 32-bit shared addresses kept in registers, position (stage, phase) kept incrementally
     // (a generic->shared conversion per wait/arrival was ~4% of this kernel's instructions at H, ncu r02)
@@ -715,12 +747,12 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
             const int u = lane >> 3, sidx = lane & 7;
             const uint32_t it = lds_u32(q1_s + 4u * (base + min(u, cnt - 1)));
             const int t = (int)(it >> 5), cl = (int)(it & 31u);
-            uint32_t x[G::CW], sc[G::CW];
-            load_row_s<G::CW>(pV_s + 4u * (t * CWV), x);
-            load_row2_s<G::CW>(stg_s + 4u * (cl * REC + (33 + sidx) * G::CW), sc);
+            uint32_t x[kCoarseWords], sc[kCoarseWords];
+            load_row_s<kCoarseWords>(pC_s + 4u * (t * kCoarseWords), x);
+            load_row_s<kCoarseWords>(stg_s + 4u * (cl * REC + C::CO + kCoarseWords * (1 + sidx)), sc);
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) x[k] -= sc[k];  // guard <=> sub-corner <= p
-            const uint32_t Ms = gather_mask<G::NG>(x);
+            for (int k = 0; k < NQ; k++) x[k] -= sc[k];  // guard <=> coarse sub-corner <= p
+            const uint32_t Ms = gather_coarse<NQ>(x);
             const uint32_t ws = lds_u32(st_s + 4u * (t * C::PS + (Ms >> 5)));
             const bool open = u < cnt && !(__funnelshift_r(ws, ws, Ms) & 1u);
             const uint32_t ob = __ballot_sync(0xffffffffu, open);
@@ -752,11 +784,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
             __syncwarp();
         };
         auto box_mask = [&](int cl) {
-            uint32_t mn[G::CW], le[G::CW];
-            load_row2_s<G::CW>(stg_s + 4u * (cl * REC + 32 * G::CW), mn);
+            uint32_t mn[kCoarseWords], le[kCoarseWords];
+            load_row_s<kCoarseWords>(stg_s + 4u * (cl * REC + C::CO), mn);
 #pragma unroll
-            for (int k = 0; k < G::CW; k++) le[k] = p[k] - mn[k];  // guard <=> corner <= p
-            return gather_mask<G::NG>(le);
+            for (int k = 0; k < NQ; k++) le[k] = p[k] - mn[k];  // guard <=> coarse corner <= p
+            return gather_coarse<NQ>(le);
         };
         const int nch_tile = (int)min((int64_t)NW, nchunks - tile * NW);
         const bool mine = (valid >> lane) & 1u;
@@ -806,7 +838,7 @@ template <int D, int MODE, int NW>
 size_t owner_smem_bytes(int tasks) {
     using C = GeoO<D, MODE, NW>;
     const size_t tpc = (size_t)tasks;
-    return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + C::PS + 1) + NW * C::QW);
+    return sizeof(uint32_t) * ((size_t)C::RING + tpc * (C::CWV + kCoarseWords + C::PS + 1) + NW * C::QW);
 }
 
 // Largest task-group count dividing NW (every group gets NW / ngrp warps) whose state fits in shared memory and
@@ -839,7 +871,7 @@ bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_owner_kernel<D, MODE, NW><<<blocks, (NW + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), ngrp, tpc,
+        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), c.cshift, ngrp, tpc,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32, c.tie.as<uint32_t>(), ext_rows32,
         c.counters.as<unsigned long long>(), host_mem, c.ext_ids.as<int32_t>());
     c.L.count++;
@@ -873,7 +905,7 @@ void launch_a(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint32_t
     const unsigned blocks = (unsigned)ceil_div(range, tpc);
     k3_mdmc_kernel<D, MODE, NW><<<blocks, (NW + 1) * 32, smem, st>>>(
         c.p_codes.as<uint32_t>(), c.p_ord.as<uint32_t>(), c.chunks_ext.as<uint32_t>(), c.q_ord.as<uint32_t>(),
-        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), tpc,
+        c.minord.as<uint32_t>(), c.nchunks_ext, j_begin, j_end, ~c.exact_mask & ((1u << D) - 1u), c.cshift, tpc,
         (c.max_level > 0 && c.max_level < D) ? c.max_level : 0, rows32,
         c.tie.as<uint32_t>(), ext_rows32, c.counters.as<unsigned long long>(), host_mem, c.ext_ids.as<int32_t>());
     c.L.count++;

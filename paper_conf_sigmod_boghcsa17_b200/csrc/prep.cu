@@ -14,6 +14,7 @@
 // bit 2 the quartile split, ... (L338 "median, then quartile, then octile").  Consecutive runs of 32
 // points in that order are "chunks" whose per-dimension minimum codes bound every member; K1 and K3
 // test a whole chunk against a task with one mask test (Eq. 1's idea, L1312) before any pair.
+#include <algorithm>
 #include <utility>
 
 #include "ctx.cuh"
@@ -64,15 +65,14 @@ __global__ void morton_kernel(const uint16_t *__restrict__ codes, const uint32_t
     perm[p] = (uint32_t)p;
 }
 
-// Chunk records (rec_rows x cw words): 32 consecutive points' code words, then the per-dimension minimum
-// code words (the chunk's lower corner), then — when rec_rows == kRecExt — the lower corners of the 8
-// sub-chunks of 4 consecutive points (the level below, K3).  One warp per chunk.
-__global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw, int rec_rows,
+// Chunk records (kRecAll x cw words, K1): 32 consecutive points' code words, then the per-dimension minimum
+// code words (the chunk's lower corner).  One warp per chunk.
+__global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw,
                                     uint32_t *__restrict__ chunks) {
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (c >= nchunks) return;
-    uint32_t *rec = chunks + c * (int64_t)(rec_rows * cw);
+    uint32_t *rec = chunks + c * (int64_t)(kRecAll * cw);
     for (int k = 0; k < cw; k++) {
         const uint32_t w = codes[(c * 32 + lane) * cw + k];
         rec[lane * cw + k] = w;
@@ -81,10 +81,58 @@ __global__ void build_chunks_kernel(const uint32_t *__restrict__ codes, int64_t 
         for (int o = 1; o < 32; o <<= 1) {
             lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
             hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
-            if (o == kSubSize / 2 && rec_rows == kRecExt && (lane & (kSubSize - 1)) == 0)
-                rec[(33 + lane / kSubSize) * cw + k] = lo | (hi << 16);  // sub-chunk corner
         }
         if (lane == 0) rec[32 * cw + k] = lo | (hi << 16);
+    }
+}
+
+// K3 chunk records (rec_ext_words(cw) words, ctx.cuh): the 32 members' code words, then the coarse lower
+// corner of the chunk and of its 8 sub-chunks of kSubSize consecutive points (the level below), four 7-bit
+// dimensions per word; padding dimensions (d..15) carry 127 (never below a task, whose padding is 0).  One warp
+// per chunk; lane i of the coarse pass owns dimension i.
+__global__ void build_chunks_ext_kernel(const uint32_t *__restrict__ codes, int64_t nchunks, int cw, int d,
+                                        uint64_t cshift, uint32_t *__restrict__ chunks) {
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (c >= nchunks) return;
+    uint32_t *rec = chunks + c * (int64_t)rec_ext_words(cw);
+    uint32_t sub_lo[kCoarseRows], sub_hi[kCoarseRows];  // row 0: chunk corner, rows 1..8: sub-chunk corners
+#pragma unroll
+    for (int r = 0; r < kCoarseRows; r++) sub_lo[r] = 0x7fffu;
+    for (int k = 0; k < cw; k++) {
+        const uint32_t w = codes[(c * 32 + lane) * cw + k];
+        rec[lane * cw + k] = w;
+        uint32_t lo = w & 0xffffu, hi = w >> 16;
+#pragma unroll
+        for (int o = 1; o < kSubSize; o <<= 1) {
+            lo = min(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+            hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+        }
+        // lane s*kSubSize holds sub-chunk s's minimum; gather the 8 sub-corners and their minimum into every lane
+        uint32_t clo = 0xffffu, chi = 0xffffu;
+#pragma unroll
+        for (int s = 0; s < 32 / kSubSize; s++) {
+            const uint32_t a = __shfl_sync(0xffffffffu, lo, s * kSubSize), b = __shfl_sync(0xffffffffu, hi, s * kSubSize);
+            if (lane == 2 * k) sub_lo[1 + s] = a;
+            if (lane == 2 * k + 1) sub_lo[1 + s] = b;
+            clo = min(clo, a);
+            chi = min(chi, b);
+        }
+        if (lane == 2 * k) sub_lo[0] = clo;
+        if (lane == 2 * k + 1) sub_lo[0] = chi;
+    }
+    // lane i < 16: the coarse corners of dimension i
+    const uint32_t sh = (uint32_t)(cshift >> (4 * (lane & 15))) & 15u;
+#pragma unroll
+    for (int r = 0; r < kCoarseRows; r++) sub_hi[r] = lane < d ? min(sub_lo[r] >> sh, 127u) : 127u;
+    // pack four dimensions per word: word g of row r = dims 4g..4g+3 (byte k = dim 4g+k)
+#pragma unroll
+    for (int r = 0; r < kCoarseRows; r++) {
+        const uint32_t v = sub_hi[r];
+        const uint32_t b1 = __shfl_down_sync(0xffffffffu, v, 1), b2 = __shfl_down_sync(0xffffffffu, v, 2),
+                       b3 = __shfl_down_sync(0xffffffffu, v, 3);
+        if (lane < 16 && (lane & 3) == 0)
+            rec[32 * cw + r * kCoarseWords + (lane >> 2)] = v | (b1 << 8) | (b2 << 16) | (b3 << 24);
     }
 }
 
@@ -204,14 +252,23 @@ __global__ void ext_build_key_kernel(const uint32_t *__restrict__ key_flag, cons
 
 inline unsigned blocks_for(int64_t n, int t) { return (unsigned)ceil_div(n > 0 ? n : 1, t); }
 
-// key of a chunk = sum of its lower-corner codes (< 2^20 for d <= 16)
-__global__ void chunk_key_kernel(const uint32_t *__restrict__ chunks, int64_t nch, int cw, int d,
+// key of a chunk = sum of its lower-corner codes (< 2^20 for d <= 16), the corner taken over the chunk's 32
+// consecutive points of the code array
+__global__ void chunk_key_kernel(const uint32_t *__restrict__ codes, int64_t nch, int cw, int d,
                                  uint64_t *__restrict__ keys, uint32_t *__restrict__ perm) {
     const int64_t ch = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (ch >= nch) return;
-    const uint32_t *mn = chunks + ch * (int64_t)(kRecExt * cw) + 32 * cw;
     uint64_t s = 0;
-    for (int i = 0; i < d; i++) s += (mn[i >> 1] >> (16 * (i & 1))) & 0xffffu;
+    for (int k = 0; k < cw; k++) {
+        uint32_t lo = 0xffffu, hi = 0xffffu;
+        for (int j = 0; j < 32; j++) {
+            const uint32_t w = codes[(ch * 32 + j) * cw + k];
+            lo = min(lo, w & 0xffffu);
+            hi = min(hi, w >> 16);
+        }
+        if (2 * k < d) s += lo;
+        if (2 * k + 1 < d) s += hi;
+    }
     keys[ch] = s;
     perm[ch] = (uint32_t)ch;
 }
@@ -341,7 +398,7 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     SKY_LAUNCH_CHECK();
     const int64_t nch = ceil_div(n, 32);
     pad_codes(c.codes_sorted.as<uint32_t>(), nch * 32, npad, cw, st, c.L);
-    build_chunks_kernel<<<blocks_for((npad / 32) * 32, 256), 256, 0, st>>>(c.codes_sorted.as<uint32_t>(), npad / 32, cw, kRecAll,
+    build_chunks_kernel<<<blocks_for((npad / 32) * 32, 256), 256, 0, st>>>(c.codes_sorted.as<uint32_t>(), npad / 32, cw,
                                                                           c.chunks_all.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
@@ -354,8 +411,15 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     SKY_LAUNCH_CHECK();
     SKY_CUDA(cudaStreamSynchronize(st));
     c.exact_mask = 0;
-    for (int i = 0; i < d; i++)
+    c.cshift = 0;
+    for (int i = 0; i < d; i++) {
         if (c.R[i] <= kCodeLevels) c.exact_mask |= 1u << i;
+        // coarse-code shift: the codes of dimension i lie in [0, min(R_i, 2^15)); shift them into 7 bits
+        const uint32_t top = std::min<uint32_t>(c.R[i], kCodeLevels) - 1u;
+        int sh = 0;
+        while ((top >> sh) > 127u) sh++;
+        c.cshift |= (uint64_t)sh << (4 * i);
+    }
     c.prepared = true;
 }
 
@@ -388,7 +452,7 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.p_ord.ensure(sizeof(uint32_t) * mm * d);
     c.q_codes.ensure(sizeof(uint16_t) * mpad * c.dp);
     c.q_ord.ensure(sizeof(uint32_t) * mpad * d);
-    c.chunks_ext.ensure(sizeof(uint32_t) * (mpad / 32) * kRecExt * cw);
+    c.chunks_ext.ensure(sizeof(uint32_t) * (mpad / 32) * rec_ext_words(cw));
     ext_build_id_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.ext_id_flag.as<uint32_t>(), c.ext_idx.as<uint32_t>(),
                                                             c.codes_id.as<uint32_t>(), c.ord.as<uint32_t>(), n, d, cw,
                                                             c.ext_ids.as<int32_t>(), c.p_codes.as<uint32_t>(),
@@ -410,11 +474,7 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     c.chunk_perm.ensure(sizeof(uint32_t) * nch);
     c.q_codes_alt.ensure(sizeof(uint32_t) * mpad * cw);
     c.q_ord_alt.ensure(sizeof(uint32_t) * mpad * d);
-    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw, kRecExt,
-                                                              c.chunks_ext.as<uint32_t>());
-    c.L.count++;
-    SKY_LAUNCH_CHECK();
-    chunk_key_kernel<<<blocks_for(nch, 256), 256, 0, st>>>(c.chunks_ext.as<uint32_t>(), nch, cw, d,
+    chunk_key_kernel<<<blocks_for(nch, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), nch, cw, d,
                                                            c.chunk_keys.as<uint64_t>(), c.chunk_perm.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
@@ -430,8 +490,8 @@ void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {
     std::swap(c.q_ord, c.q_ord_alt);
     pad_codes(c.q_codes.as<uint32_t>(), nch * 32, mpad, cw, st, c.L);
     pad_ord(c.q_ord.as<uint32_t>(), nch * 32, mpad, d, st, c.L);
-    build_chunks_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw, kRecExt,
-                                                              c.chunks_ext.as<uint32_t>());
+    build_chunks_ext_kernel<<<blocks_for(mpad, 256), 256, 0, st>>>(c.q_codes.as<uint32_t>(), mpad / 32, cw, d, c.cshift,
+                                                                  c.chunks_ext.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     c.nchunks_ext = nch;
