@@ -793,6 +793,22 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
         const int nch_tile = (int)min((int64_t)NW, nchunks - tile * NW);
         const bool mine = (valid >> lane) & 1u;
         int cl = wsub;
+        // four chunks per iteration where a warp has that many in the tile (ILP; H K3 79.9 -> 79.2 ms), then pairs
+        for (; cl + 3 * wpg < nch_tile; cl += 4 * wpg) {
+            const uint32_t M0 = box_mask(cl), M1 = box_mask(cl + wpg), M2 = box_mask(cl + 2 * wpg), M3 = box_mask(cl + 3 * wpg);
+            const uint32_t w0 = lds_u32(st_own + 4u * (M0 >> 5)), w1 = lds_u32(st_own + 4u * (M1 >> 5));
+            const uint32_t w2 = lds_u32(st_own + 4u * (M2 >> 5)), w3 = lds_u32(st_own + 4u * (M3 >> 5));
+            const uint32_t todo0 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w0, w0, M0) & 1u));
+            const uint32_t todo1 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w1, w1, M1) & 1u));
+            const uint32_t todo2 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w2, w2, M2) & 1u));
+            const uint32_t todo3 = __ballot_sync(0xffffffffu, mine && !(__funnelshift_r(w3, w3, M3) & 1u));
+            n_box += 4 * __popc(valid);
+            if ((todo0 | todo1 | todo2 | todo3) == 0) continue;
+            enqueue(todo0, cl);
+            enqueue(todo1, cl + wpg);
+            enqueue(todo2, cl + 2 * wpg);
+            enqueue(todo3, cl + 3 * wpg);
+        }
         for (; cl + wpg < nch_tile; cl += 2 * wpg) {
             const uint32_t M0 = box_mask(cl), M1 = box_mask(cl + wpg);
             const uint32_t w0 = lds_u32(st_own + 4u * (M0 >> 5)), w1 = lds_u32(st_own + 4u * (M1 >> 5));
