@@ -299,11 +299,12 @@ def test_global_tie_rows_d16(tuning):
 
 
 @pytest.mark.parametrize("warps", [16, 24])
-@pytest.mark.parametrize("case", [("ct", 6000, 10, 921), ("I", 5000, 8, 922), ("grid", 3000, 12, 923)])
+@pytest.mark.parametrize("case", [("ct", 6000, 10, 921), ("I", 5000, 8, 922), ("grid", 3000, 12, 923),
+                                  ("A", 7000, 12, 924)])
 def test_k3_design_o_warp_counts(tuning, warps, case):
-    """Design O (task-owner warps, the tie-exact state) with 16 and with 24 consumer warps: tiles of 16 or 24
+    """Design O (task-owner warps) with 16 and 24 consumer warps: tiles of 16 or 24
     chunks, group counts dividing the warp count (e.g. 3 groups of 8 warps), queue items carrying a chunk index
-    up to 23; both must equal the oracle."""
+    up to 23; all must equal the oracle."""
     tuning("k3_warps", warps)
     tuning("k3_design", "O")
     dist, n, d, seed = case
