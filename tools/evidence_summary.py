@@ -113,9 +113,16 @@ def main():
         md += ["## Launch list of the default bench (H), `ncu --metrics gpu__time_duration.sum --clock-control none`",
                "", ncu_summary.launches(dst).replace(ROOT + "/", ""), ""]
     md += ["## `ncu --set full` captures (one launch each)", ""]
-    for rep in sorted(glob.glob(os.path.join(OUT, "ev_prof_*.ncu-rep"))):
+    caps = sorted(glob.glob(os.path.join(OUT, "ev_prof_*.ncu-rep")))
+    have = {c[:-len(".ncu-rep")] for c in caps}
+    caps += [c for c in sorted(glob.glob(os.path.join(OUT, "ev_prof_*.raw.csv"))) if c[:-len(".raw.csv")] not in have]
+    for rep in caps:
         md += [ncu_summary.report(rep).replace(ROOT + "/", "").replace("gpurun_out/", ""), ""]
-        if "k3_mdmc_H" in rep or "k3_owner" in rep:
+        base = rep[:-len(".ncu-rep")] if rep.endswith(".ncu-rep") else rep[:-len(".raw.csv")]
+        if os.path.exists(base + ".lines.txt"):  # per-source-line instructions / stall samples (tools/ncu_lines.py)
+            md += ["Hottest source lines (`tools/ncu_lines.py`: share of executed warp instructions, share of "
+                   "warp-stall samples):", "", "```", open(base + ".lines.txt").read().strip(), "```", ""]
+        elif rep.endswith(".ncu-rep") and "k3_" in rep:
             md += ["Hottest source lines:", "", k3_passes(rep), ""]
     with open(os.path.join(PROF, f"{tag}_ncu_summary.md"), "w") as fo:
         fo.write("\n".join(md) + "\n")
