@@ -860,10 +860,27 @@ size_t owner_smem_bytes(int tasks) {
 // Largest task-group count dividing NW (every group gets NW / ngrp warps) whose state fits in shared memory and
 // that does not exceed `want`; 0 if not even one group fits.
 template <int D, int MODE, int NW>
-int owner_groups(int64_t want) {
-    int best = 0;
+int owner_groups(int64_t want, int64_t range, int num_sms) {
+    // candidates: group counts dividing NW that fit, at most `want` (>= one CTA per SM for small ranges).  The
+    // largest one, unless the range is under 4 waves of such CTAs -- a shard of S+ at N > 1 ranks: H / 8 = 88K
+    // tasks are 2.3 waves of 8-group CTAs -- where the count minimising waves x (groups + 1) keeps the last wave
+    // from leaving most SMs idle (H / 8: 4 groups, K3 12.7 -> 11.6 ms).  Over many waves the CTA durations vary
+    // enough to smooth the tail, and fewer groups only cost more chunk-stream passes (C3A, 10 waves: 6 instead
+    // of 8 groups measured 32.4 -> 40.5 ms).
+    int gmax = 0;
     for (int g = 1; g <= NW; g++)
-        if (NW % g == 0 && owner_smem_bytes<D, MODE, NW>(g * 32) <= (size_t)kSmemBytes && (g == 1 || g <= want)) best = g;
+        if (NW % g == 0 && owner_smem_bytes<D, MODE, NW>(g * 32) <= (size_t)kSmemBytes && (g == 1 || g <= want)) gmax = g;
+    if (gmax < 1 || ceil_div(range, (int64_t)gmax * 32) >= 4 * (int64_t)num_sms) return gmax;
+    int best = gmax;
+    int64_t best_cost = ceil_div(ceil_div(range, (int64_t)gmax * 32), (int64_t)num_sms) * (gmax + 1);
+    for (int g = gmax - 1; g >= 1; g--) {
+        if (NW % g != 0) continue;
+        const int64_t cost = ceil_div(ceil_div(range, (int64_t)g * 32), (int64_t)num_sms) * (g + 1);
+        if (cost < best_cost) {
+            best = g;
+            best_cost = cost;
+        }
+    }
     return best;
 }
 
@@ -873,7 +890,7 @@ bool launch_owner(Ctx &c, int64_t j_begin, int64_t j_end, uint32_t *rows32, uint
     const int64_t range = j_end - j_begin;
     // groups per CTA: the shared-memory budget, but at least one CTA per SM for small ranges
     const int64_t want = std::max<int64_t>(1, ceil_div(ceil_div(range, c.num_sms), 32));
-    int ngrp = owner_groups<D, MODE, NW>(want), tpc = ngrp * 32;
+    int ngrp = owner_groups<D, MODE, NW>(want, range, c.num_sms), tpc = ngrp * 32;
     if (ngrp < 1) {
         // one partial group: as many tasks as the shared memory holds (d = 16: 22 tasks of 8 KB state)
         ngrp = 1;
