@@ -39,7 +39,7 @@ constexpr int stages_for() { return CW <= 6 ? 6 : 4; }
 template <int CW>
 __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
     const uint32_t *__restrict__ chunks, const uint32_t *__restrict__ supers, const uint32_t *__restrict__ ord_sorted,
-    int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset, int64_t blk_step,
+    int64_t n, int d, uint32_t inexact, int64_t nchunks, int64_t blk_offset, int64_t blk_step, int nsplit,
     uint8_t *__restrict__ ext_sorted, unsigned long long *__restrict__ counters) {
     constexpr int REC = 33 * CW;        // chunk record words: 32 code rows, then the lower corner
     constexpr int CWS = (CW + 3) & ~3;  // tile-corner record words
@@ -53,7 +53,10 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
     volatile int32_t *tile_idx = reinterpret_cast<volatile int32_t *>(pV + kTasks * CWV);  // [kStages]
     uint32_t *ucorner = pV + kTasks * CWV + kStages;   // [kWarps][CW] upper corner of each warp's tasks
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int64_t blk = blk_offset + (int64_t)blockIdx.x * blk_step;
+    // CTA = (block of kTasks tree positions, split of the competitor tiles): with nsplit > 1 the CTAs of a block
+    // stream the tiles t = split (mod nsplit) each, and a task is outside S+ iff some split finds a dominator
+    const int64_t blk = blk_offset + (int64_t)(blockIdx.x / nsplit) * blk_step;
+    const int split = (int)(blockIdx.x % nsplit);
     const int64_t s0 = blk * kTasks;
     const int64_t ntiles = ceil_div_dev(nchunks, kTileChunks);
 
@@ -109,7 +112,7 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
         for (int64_t t0 = 0; t0 < ntiles; t0 += 32) {
             const int64_t t = t0 + lane;
             bool pass = false;
-            if (t < ntiles) {
+            if (t < ntiles && (int)(t % nsplit) == split) {
                 const uint32_t *sc = supers + t * CWS;
                 uint32_t acc = 0xffffffffu;
 #pragma unroll
@@ -209,7 +212,17 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2) k1_prefilter_kernel(
         atomicAdd(&counters[0], n_box);
         atomicAdd(&counters[1], n_pair);
     }
-    if (ps < n) ext_sorted[ps] = (live >> lane) & 1u;
+    // nsplit == 1: the flag; else the block's flags were set to 1 before the launch and a split clears the tasks it
+    // found dominated (plain byte stores of 0: idempotent across splits)
+    if (ps < n && (nsplit == 1 || !((live >> lane) & 1u))) ext_sorted[ps] = (live >> lane) & 1u;
+}
+
+// ext[ps] = 1 for the tree positions of the blocks b = off (mod step) (the splits then clear the dominated ones)
+__global__ void k1_fill_kernel(int64_t n, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uint8_t *ext) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nblk_mine * kTasks) return;
+    const int64_t ps = (blk_offset + (i / kTasks) * blk_step) * kTasks + (i % kTasks);
+    if (ps < n) ext[ps] = 1u;
 }
 
 template <int CW>
@@ -219,9 +232,20 @@ void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uin
                                             (size_t)kTasks * ((CW + 3) & ~3) + kStages + (size_t)kWarps * CW);
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
-    k1_prefilter_kernel<CW><<<(unsigned)nblk_mine, (kWarps + 1) * 32, smem, st>>>(
+    // Splits of the competitor stream when the rank's blocks fill fewer than 4 waves (two CTAs per SM): a rank's
+    // K1 time is its slowest CTA, and at N = 8 ranks the 245 blocks of H are under one wave (K1 4.1 ms per rank
+    // against 13.0 ms on one GPU); more, shorter CTAs spread it (a task's early exit then only covers its split)
+    const int64_t slots = 2 * (int64_t)c.num_sms;
+    const int nsplit = (int)std::min<int64_t>(8, std::max<int64_t>(1, ceil_div(4 * slots, nblk_mine)));
+    if (nsplit > 1) {
+        k1_fill_kernel<<<(unsigned)ceil_div(nblk_mine * kTasks, 256), 256, 0, st>>>(c.n, blk_offset, blk_step, nblk_mine,
+                                                                               ext);
+        c.L.count++;
+        SKY_LAUNCH_CHECK();
+    }
+    k1_prefilter_kernel<CW><<<(unsigned)(nblk_mine * nsplit), (kWarps + 1) * 32, smem, st>>>(
         c.chunks_all.as<uint32_t>(), c.supers_all.as<uint32_t>(), c.ord_sorted.as<uint32_t>(), c.n, c.d, inexact,
-        c.nchunks_all, blk_offset, blk_step, ext, c.counters.as<unsigned long long>());
+        c.nchunks_all, blk_offset, blk_step, nsplit, ext, c.counters.as<unsigned long long>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
 }
