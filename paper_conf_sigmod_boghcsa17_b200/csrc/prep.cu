@@ -384,7 +384,9 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     }
     SKY_CUDA(cudaMemcpyAsync(c.R, c.rbuf.p, sizeof(uint32_t) * d, cudaMemcpyDeviceToHost, st));
     // static-tree leaf order: Morton key of the codes (top bits first), then chunks of 32
-    const int bits_per_dim = std::min(15, 64 / d);
+    // (at most 32 key bits: the top bits decide the chunks of 32 and their sub-chunks -- 2^15 chunks at n = 1M --
+    // and the stable sort keeps id order below; 32 bits sort in 4 radix passes instead of 8)
+    const int bits_per_dim = std::min(15, 32 / d);
     morton_kernel<<<blocks_for(n, 256), 256, 0, st>>>(c.codes_id.as<uint16_t>(), c.rbuf.as<uint32_t>(), n, d, c.dp,
                                                       bits_per_dim, c.keysum.as<uint64_t>(), c.perm.as<uint32_t>());
     c.L.count++;
