@@ -232,11 +232,15 @@ void launch(Ctx &c, int64_t blk_offset, int64_t blk_step, int64_t nblk_mine, uin
                                             (size_t)kTasks * ((CW + 3) & ~3) + kStages + (size_t)kWarps * CW);
     SKY_CUDA(cudaFuncSetAttribute(k1_prefilter_kernel<CW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     const uint32_t inexact = ~c.exact_mask & ((1u << c.d) - 1u);
-    // Splits of the competitor stream when the rank's blocks fill fewer than 4 waves (two CTAs per SM): a rank's
+    // Splits of the competitor stream when the rank's blocks fill fewer than 8 waves (two CTAs per SM): a rank's
     // K1 time is its slowest CTA, and at N = 8 ranks the 245 blocks of H are under one wave (K1 4.1 ms per rank
-    // against 13.0 ms on one GPU); more, shorter CTAs spread it (a task's early exit then only covers its split)
+    // against 13.0 ms on one GPU); more, shorter CTAs spread it (a task's early exit then only covers its split).
+    // Per-rank K1 at N = 8: H 4.1 -> 3.0 (4 waves) -> 2.7 ms (8 waves), C4 9.2 -> 5.8 -> 4.1 ms; one GPU unchanged.
     const int64_t slots = 2 * (int64_t)c.num_sms;
-    const int nsplit = (int)std::min<int64_t>(8, std::max<int64_t>(1, ceil_div(4 * slots, nblk_mine)));
+#ifndef SKY_K1_WAVES
+#define SKY_K1_WAVES 8
+#endif
+    const int nsplit = (int)std::min<int64_t>(16, std::max<int64_t>(1, ceil_div(SKY_K1_WAVES * slots, nblk_mine)));
     if (nsplit > 1) {
         k1_fill_kernel<<<(unsigned)ceil_div(nblk_mine * kTasks, 256), 256, 0, st>>>(c.n, blk_offset, blk_step, nblk_mine,
                                                                                ext);
