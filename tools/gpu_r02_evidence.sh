@@ -26,12 +26,17 @@ summ() {
 }
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_launches_H.csv \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu > gpurun_out/ev_ncu_launch.log 2>&1
+if [ "${NCU_K3:-1}" = 1 ]; then
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k3_ -c 1 -f -o gpurun_out/ev_prof_k3_H \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k3_H.log 2>&1
 summ ev_prof_k3_H keep
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k3_ -c 1 -f -o gpurun_out/ev_prof_k3_C4 \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config C4 > gpurun_out/ev_ncu_k3_C4.log 2>&1
 summ ev_prof_k3_C4
+fi
+# per-rank K1 / K3 work of an N-GPU run, measured on this one GPU (tools/k3_shard_time.py)
+for c in ${SHARD_CONFIGS:-H C4}; do for w in 1 2 4 8; do timeout 900 python tools/k3_shard_time.py $c $w 3; done; done \
+  > gpurun_out/ev_shards.jsonl 2> gpurun_out/ev_shards.err
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:k1_ -c 1 -f -o gpurun_out/ev_prof_k1_H \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k1_H.log 2>&1
 summ ev_prof_k1_H
