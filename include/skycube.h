@@ -182,6 +182,24 @@ void skycube_ctx_destroy(skycube_ctx *ctx);
  * d_points: [n*d] float32 row-major on the device. */
 skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, void *stream);
 
+/* The two halves of skycube_dev_prepare, for a preparation sharded over the ranks of a multi-GPU run (SURVEY
+ * §8(e); the per-dimension ranks of K2 are independent across dimensions, so rank r computes the codes of its
+ * slice of the dimensions and the ranks all-gather them):
+ *
+ * skycube_dev_prepare_dims: K0 (validation, order-preserving keys of EVERY dimension, kept in the context) and
+ *   K2 on the dimensions [dim_begin, dim_end) only: d_codes_dm (device, uint16 [dim_end - dim_begin][n],
+ *   dim-major, caller-owned) receives their 15-bit codes; d_R / d_minord (device, uint32 [d], caller-owned)
+ *   receive, at the indices dim_begin .. dim_end - 1, the number of distinct values and the minimum order key
+ *   of each dimension.  dim_begin == dim_end runs K0 only.  Errors as skycube_dev_prepare (ENAN on NaN).
+ * skycube_dev_prepare_finish: completes the preparation from every dimension's codes: d_codes_dm uint16
+ *   [d][n] (dim-major), d_R and d_minord uint32 [d], all device and caller-owned (read only).  Afterwards the
+ *   context is in the state skycube_dev_prepare leaves it in.  EINVAL before skycube_dev_prepare_dims. */
+skycube_status skycube_dev_prepare_dims(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, int32_t dim_begin,
+                                        int32_t dim_end, uint16_t *d_codes_dm, uint32_t *d_R, uint32_t *d_minord,
+                                        void *stream);
+skycube_status skycube_dev_prepare_finish(skycube_ctx *ctx, const uint16_t *d_codes_dm, const uint32_t *d_R,
+                                          const uint32_t *d_minord, void *stream);
+
 /* Phase 2: extended-skyline prefilter (K1).  The prepared (static-tree) positions are cut into blocks of
  * 512 (one K1 CTA each); this call processes the blocks b with b % tile_step == tile_offset (interleaving balances ranks).
  * Writes d_ext_sorted[s] = 1 iff the point at prepared position s is in S+(P), 0 otherwise, for the

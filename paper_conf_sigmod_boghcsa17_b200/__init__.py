@@ -27,6 +27,7 @@ EXPORTED = (
     "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_free",
     "skycube_hashcube_query", "skycube_ctx_set_max_level", "skycube_dev_hashcube", "skycube_build_sdsc",
     "skycube_set_tuning", "skycube_dev_lattice_count", "skycube_dev_lattice_scatter", "skycube_dev_membership",
+    "skycube_dev_prepare_dims", "skycube_dev_prepare_finish",
 )
 
 
@@ -98,6 +99,8 @@ def lib():
         L.skycube_ctx_destroy.argtypes = [P]
         L.skycube_ctx_destroy.restype = None
         L.skycube_dev_prepare.argtypes = [P, P, I64, I32, P]
+        L.skycube_dev_prepare_dims.argtypes = [P, P, I64, I32, I32, I32, P, P, P, P]
+        L.skycube_dev_prepare_finish.argtypes = [P, P, P, P, P]
         L.skycube_dev_prefilter.argtypes = [P, I64, I64, P, P]
         L.skycube_dev_set_ext.argtypes = [P, P, ctypes.POINTER(I64), P]
         L.skycube_dev_mdmc.argtypes = [P, I64, I64, P, P, P]
@@ -121,6 +124,7 @@ def lib():
         L.skycube_dev_lattice_scatter.argtypes = [P, P, I64, I64, P, I32, I32, P, P, ctypes.POINTER(I64), P]
         L.skycube_dev_membership.argtypes = [P, P, I64, I64, I64, I64, P, P]
         for f in ("skycube_dev_lattice_count", "skycube_dev_lattice_scatter", "skycube_dev_membership",
+                  "skycube_dev_prepare_dims", "skycube_dev_prepare_finish",
                   "skycube_set_tuning", "skycube_build", "skycube_build_ex", "skycube_ctx_create", "skycube_dev_prepare",
                   "skycube_dev_prefilter", "skycube_dev_set_ext", "skycube_dev_mdmc", "skycube_dev_compact",
                   "skycube_ctx_info", "skycube_ctx_counters", "skycube_build_hashcube", "skycube_hashcube_query",
@@ -369,6 +373,14 @@ class Context:
 
     def prepare(self, d_points: int, n: int, d: int, stream: int = 0):
         _check(lib().skycube_dev_prepare(self._h, d_points, n, d, stream or None))
+
+    def prepare_dims(self, d_points: int, n: int, d: int, dim_begin: int, dim_end: int, d_codes_dm: int, d_R: int,
+                     d_minord: int, stream: int = 0):
+        _check(lib().skycube_dev_prepare_dims(self._h, d_points, n, d, dim_begin, dim_end, d_codes_dm or None,
+                                              d_R or None, d_minord or None, stream or None))
+
+    def prepare_finish(self, d_codes_dm: int, d_R: int, d_minord: int, stream: int = 0):
+        _check(lib().skycube_dev_prepare_finish(self._h, d_codes_dm, d_R, d_minord, stream or None))
 
     def prefilter(self, d_ext_sorted: int, tile_offset: int = 0, tile_step: int = 1, stream: int = 0):
         _check(lib().skycube_dev_prefilter(self._h, tile_offset, tile_step, d_ext_sorted, stream or None))

@@ -813,7 +813,7 @@ void skycube_ctx_destroy(skycube_ctx *ctx) {
     cudaSetDevice(ctx->c.device);
     sky::Ctx &c = ctx->c;
     for (sky::DevBuf *b : {&c.ord, &c.keysum, &c.perm, &c.comp_keys, &c.comp_vals, &c.keys_alt, &c.vals_alt,
-                           &c.counts, &c.scan_tmp, &c.flags, &c.scanned, &c.rbuf, &c.minord, &c.nanflag, &c.codes_id,
+                           &c.counts, &c.scan_tmp, &c.flags, &c.scanned, &c.rbuf, &c.minord, &c.nanflag, &c.codes_dm, &c.codes_id,
                            &c.codes_sorted, &c.ord_sorted, &c.ext_id_flag, &c.ext_idx, &c.key_flag, &c.key_idx,
                            &c.ext_ids, &c.p_codes, &c.p_ord, &c.q_codes, &c.q_ord, &c.tie, &c.lat_counts,
                            &c.scan64_tmp, &c.chunks_all, &c.chunks_ext, &c.supers_all, &c.counters, &ctx->input, &ctx->ext8, &ctx->rows32, &ctx->ext_rows32,
@@ -854,6 +854,32 @@ skycube_status skycube_dev_prepare(skycube_ctx *ctx, const float *d_points, int6
     return guarded([&] {
         SKY_CUDA(cudaSetDevice(ctx->c.device));
         sky::prep_run(ctx->c, d_points, n, d, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_prepare_dims(skycube_ctx *ctx, const float *d_points, int64_t n, int32_t d, int32_t dim_begin,
+                                        int32_t dim_end, uint16_t *d_codes_dm, uint32_t *d_R, uint32_t *d_minord,
+                                        void *stream) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (d < 1 || d > 16) return fail(SKYCUBE_EINVAL, "d must be in [1, 16]");
+    if (n < 1 || n > INT32_MAX) return fail(SKYCUBE_EINVAL, "n must be in [1, INT32_MAX]");
+    if (dim_begin < 0 || dim_end < dim_begin || dim_end > d) return fail(SKYCUBE_EINVAL, "bad dimension slice");
+    if (!d_points || (dim_end > dim_begin && (!d_codes_dm || !d_R || !d_minord)))
+        return fail(SKYCUBE_EINVAL, "NULL buffer");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::prep_dims(ctx->c, d_points, n, d, dim_begin, dim_end, d_codes_dm, d_R, d_minord, (cudaStream_t)stream);
+    });
+}
+
+skycube_status skycube_dev_prepare_finish(skycube_ctx *ctx, const uint16_t *d_codes_dm, const uint32_t *d_R,
+                                          const uint32_t *d_minord, void *stream) {
+    if (!ctx) return fail(SKYCUBE_EINVAL, "ctx == NULL");
+    if (ctx->c.n < 1 || ctx->c.d < 1) return fail(SKYCUBE_EINVAL, "skycube_dev_prepare_finish before skycube_dev_prepare_dims");
+    if (!d_codes_dm || !d_R || !d_minord) return fail(SKYCUBE_EINVAL, "NULL buffer");
+    return guarded([&] {
+        SKY_CUDA(cudaSetDevice(ctx->c.device));
+        sky::prep_finish(ctx->c, d_codes_dm, d_R, d_minord, (cudaStream_t)stream);
     });
 }
 

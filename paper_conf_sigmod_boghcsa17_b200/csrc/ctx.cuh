@@ -74,6 +74,7 @@ struct Ctx {
     DevBuf rbuf;        // u32 [kMaxD]
     DevBuf minord;      // u32 [kMaxD]  key of each dimension's minimum value
     DevBuf nanflag;     // u32 [1]
+    DevBuf codes_dm;    // u16 [d][n]  codes, dim-major (prep_dims output on one GPU)
     DevBuf codes_id;    // u16 [n*dp]  id order
     DevBuf codes_sorted;// u16 [npad*dp]  static-tree (Morton) order, padded to whole chunk tiles
     DevBuf ord_sorted;  // u32 [n*d]      static-tree order
@@ -107,6 +108,11 @@ struct Ctx {
 
 // prep.cu
 void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st);
+// the two halves of prep_run (multi-GPU prepare: every rank the codes of a slice of the dimensions, then an
+// all-gather of the codes, then prep_finish on every rank)
+void prep_dims(Ctx &c, const float *d_points, int64_t n, int d, int db, int de, uint16_t *codes_dm, uint32_t *R,
+               uint32_t *minord, cudaStream_t st);
+void prep_finish(Ctx &c, const uint16_t *codes_dm, const uint32_t *R, const uint32_t *minord, cudaStream_t st);
 void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st);
 void or_flags(Ctx &c, const uint8_t *stage, int k, int64_t n, uint8_t *out, cudaStream_t st);
 // k1_prefilter.cu

@@ -29,10 +29,11 @@ __device__ __forceinline__ uint32_t ord_key(float x) {
     return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
 }
 
-// K0: one thread per point.
-__global__ void k0_canon_kernel(const float *__restrict__ pts, int64_t n, int d, uint32_t *__restrict__ ord,
-                                uint64_t *__restrict__ comp_keys, uint32_t *__restrict__ comp_vals,
-                                uint32_t *__restrict__ nanflag) {
+// K0: one thread per point: order-preserving keys of every dimension, and the (dimension, key) sort items of the
+// dimensions [db, de) (all of them on one GPU; a slice per rank in the multi-GPU prepare), local index i - db.
+__global__ void k0_canon_kernel(const float *__restrict__ pts, int64_t n, int d, int db, int de,
+                                uint32_t *__restrict__ ord, uint64_t *__restrict__ comp_keys,
+                                uint32_t *__restrict__ comp_vals, uint32_t *__restrict__ nanflag) {
     const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
     bool nan = false;
@@ -41,8 +42,10 @@ __global__ void k0_canon_kernel(const float *__restrict__ pts, int64_t n, int d,
         nan |= (x != x);
         const uint32_t o = ord_key(x);
         ord[p * d + i] = o;
-        comp_keys[(int64_t)i * n + p] = ((uint64_t)i << 32) | o;
-        comp_vals[(int64_t)i * n + p] = (uint32_t)p;
+        if (i >= db && i < de) {
+            comp_keys[(int64_t)(i - db) * n + p] = ((uint64_t)(i - db) << 32) | o;
+            comp_vals[(int64_t)(i - db) * n + p] = (uint32_t)p;
+        }
     }
     if (nan) atomicOr(nanflag, 1u);
 }
@@ -180,9 +183,10 @@ __global__ void k2_distinct_kernel(const uint32_t *__restrict__ ex, const uint32
 
 // code = dense rank if the dimension has <= 2^15 distinct values, else floor(rank * 2^15 / R):
 // monotone in the value and equal for equal values (Λ3); injective iff R <= 2^15.
+// codes of the slice's dimensions, dim-major: codes_dm[i][p] (i local); R indexed by local dimension
 __global__ void k2_codes_kernel(const uint32_t *__restrict__ ex, const uint32_t *__restrict__ flags,
                                 const uint32_t *__restrict__ comp_vals, const uint32_t *__restrict__ R,
-                                int64_t n, int64_t total, int dp, uint16_t *__restrict__ codes) {
+                                int64_t n, int64_t total, uint16_t *__restrict__ codes_dm) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= total) return;
     const int dim = (int)(t / n);
@@ -190,14 +194,16 @@ __global__ void k2_codes_kernel(const uint32_t *__restrict__ ex, const uint32_t 
     const uint32_t rank = (ex[t] + flags[t]) - (ex[a] + flags[a]);
     const uint32_t r = R[dim];
     const uint32_t code = r <= kCodeLevels ? rank : (uint32_t)(((uint64_t)rank * kCodeLevels) / r);
-    codes[(int64_t)comp_vals[t] * dp + dim] = (uint16_t)code;
+    codes_dm[(int64_t)dim * n + comp_vals[t]] = (uint16_t)code;
 }
 
-// Padding dimensions d..dp-1 carry code 1 on the competitor side (the task side zeroes them).
-__global__ void k2_pad_kernel(int64_t n, int d, int dp, uint16_t *__restrict__ codes) {
+// codes_id[p][i] = codes_dm[i][p] for i < d; padding dimensions d..dp-1 carry code 1 on the competitor side
+// (the task side zeroes them)
+__global__ void k2_transpose_kernel(const uint16_t *__restrict__ codes_dm, int64_t n, int d, int dp,
+                                    uint16_t *__restrict__ codes) {
     const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= n) return;
-    for (int i = d; i < dp; i++) codes[p * dp + i] = 1;
+    for (int i = 0; i < dp; i++) codes[p * dp + i] = i < d ? codes_dm[(int64_t)i * n + p] : (uint16_t)1;
 }
 
 __global__ void gather_sorted_kernel(const uint32_t *__restrict__ perm, const uint32_t *__restrict__ codes_id,
@@ -321,7 +327,11 @@ void or_flags(Ctx &c, const uint8_t *stage, int k, int64_t n, uint8_t *out, cuda
     SKY_LAUNCH_CHECK();
 }
 
-void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) {
+// K0 + K2 on the dimensions [db, de): order-preserving keys of every dimension (c.ord), and for the slice the
+// dense-rank codes (dim-major, codes_dm[i - db][p]), distinct-value counts R[i] and minimum keys minord[i]
+// (arrays indexed by global dimension; only the slice's entries are written).  One GPU: the whole range.
+void prep_dims(Ctx &c, const float *d_points, int64_t n, int d, int db, int de, uint16_t *codes_dm, uint32_t *R,
+               uint32_t *minord, cudaStream_t st) {
     c.n = n;
     c.d = d;
     c.dp = dpad_of(d);
@@ -329,59 +339,77 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
     c.prepared = false;
     c.ext_ready = false;
     c.m = 0;
-    const int64_t nd = n * d;
-    const int cw = c.dp / 2;  // 32-bit code words per point
-    const int64_t npad = ceil_div(n, 32) * 32 + kChunkTilePad;  // whole chunks + whole chunk tiles
-    c.ord.ensure(sizeof(uint32_t) * nd);
-    c.keysum.ensure(sizeof(uint64_t) * n);
-    c.perm.ensure(sizeof(uint32_t) * n);
+    const int nl = de - db;
+    const int64_t nd = n * (nl > 0 ? nl : 1);
+    c.ord.ensure(sizeof(uint32_t) * n * d);
     c.comp_keys.ensure(sizeof(uint64_t) * nd);
     c.comp_vals.ensure(sizeof(uint32_t) * nd);
-    c.keys_alt.ensure(sizeof(uint64_t) * nd);
-    c.vals_alt.ensure(sizeof(uint32_t) * nd);
-    c.counts.ensure(sizeof(uint32_t) * radix_scratch_counts(nd));
-    c.scan_tmp.ensure(scan_tmp_bytes((int64_t)radix_scratch_counts(nd) > nd ? (int64_t)radix_scratch_counts(nd) : nd));
+    c.keys_alt.ensure(sizeof(uint64_t) * std::max<int64_t>(nd, n));
+    c.vals_alt.ensure(sizeof(uint32_t) * std::max<int64_t>(nd, n));
+    const int64_t cnt = std::max<int64_t>(radix_scratch_counts(nd), radix_scratch_counts(n));
+    c.counts.ensure(sizeof(uint32_t) * cnt);
+    c.scan_tmp.ensure(scan_tmp_bytes(std::max<int64_t>(cnt, nd)));
     c.flags.ensure(sizeof(uint32_t) * nd);
     c.scanned.ensure(sizeof(uint32_t) * nd);
-    c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
-    c.minord.ensure(sizeof(uint32_t) * kMaxD);
     c.nanflag.ensure(sizeof(uint32_t));
-    c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
-    c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
-    c.ord_sorted.ensure(sizeof(uint32_t) * npad * d);
-    c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * kRecAll * cw);
 
     SKY_CUDA(cudaMemsetAsync(c.nanflag.p, 0, sizeof(uint32_t), st));
-    k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, c.ord.as<uint32_t>(), c.comp_keys.as<uint64_t>(),
-                                                        c.comp_vals.as<uint32_t>(), c.nanflag.as<uint32_t>());
+    k0_canon_kernel<<<blocks_for(n, 256), 256, 0, st>>>(d_points, n, d, db, de, c.ord.as<uint32_t>(),
+                                                        c.comp_keys.as<uint64_t>(), c.comp_vals.as<uint32_t>(),
+                                                        c.nanflag.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     uint32_t nan = 0;
     SKY_CUDA(cudaMemcpyAsync(&nan, c.nanflag.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
     SKY_CUDA(cudaStreamSynchronize(st));
     if (nan) throw Error{2, "NaN in input points"};
+    if (nl <= 0) return;
 
     // K2: per-dimension sort of (dim, key) -> dense ranks -> codes.
-    radix_sort_u64(c.comp_keys.as<uint64_t>(), c.comp_vals.as<uint32_t>(), nd, 36, c.keys_alt.as<uint64_t>(),
+    int dbits = 0;
+    while ((1 << dbits) < nl) dbits++;
+    radix_sort_u64(c.comp_keys.as<uint64_t>(), c.comp_vals.as<uint32_t>(), nd, 32 + dbits, c.keys_alt.as<uint64_t>(),
                    c.vals_alt.as<uint32_t>(), c.counts.as<uint32_t>(), c.scan_tmp.p, st, c.L);
     k2_flags_kernel<<<blocks_for(nd, 256), 256, 0, st>>>(c.comp_keys.as<uint64_t>(), n, nd, c.flags.as<uint32_t>());
     c.L.count++;
     SKY_LAUNCH_CHECK();
     exclusive_scan_u32(c.flags.as<uint32_t>(), c.scanned.as<uint32_t>(), nd, c.scan_tmp.p, st, c.L);
     k2_distinct_kernel<<<1, 32, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(), c.comp_keys.as<uint64_t>(), n,
-                                         d, c.rbuf.as<uint32_t>(), c.minord.as<uint32_t>());
+                                         nl, R + db, minord + db);
     c.L.count++;
     SKY_LAUNCH_CHECK();
     k2_codes_kernel<<<blocks_for(nd, 256), 256, 0, st>>>(c.scanned.as<uint32_t>(), c.flags.as<uint32_t>(),
-                                                         c.comp_vals.as<uint32_t>(), c.rbuf.as<uint32_t>(), n, nd,
-                                                         c.dp, c.codes_id.as<uint16_t>());
+                                                         c.comp_vals.as<uint32_t>(), R + db, n, nd, codes_dm);
     c.L.count++;
     SKY_LAUNCH_CHECK();
-    if (c.dp > d) {
-        k2_pad_kernel<<<blocks_for(n, 256), 256, 0, st>>>(n, d, c.dp, c.codes_id.as<uint16_t>());
-        c.L.count++;
-        SKY_LAUNCH_CHECK();
-    }
+}
+
+// The rest of the preparation from every dimension's codes (dim-major codes_dm[d][n], R[d], minord[d], device):
+// codes by id, the static-tree (Morton) order, chunk records and tile corners (K1 competitors).
+void prep_finish(Ctx &c, const uint16_t *codes_dm, const uint32_t *R, const uint32_t *minord, cudaStream_t st) {
+    const int64_t n = c.n;
+    const int d = c.d;
+    const int cw = c.dp / 2;  // 32-bit code words per point
+    const int64_t npad = ceil_div(n, 32) * 32 + kChunkTilePad;  // whole chunks + whole chunk tiles
+    c.keysum.ensure(sizeof(uint64_t) * n);
+    c.perm.ensure(sizeof(uint32_t) * n);
+    c.keys_alt.ensure(sizeof(uint64_t) * n);
+    c.vals_alt.ensure(sizeof(uint32_t) * n);
+    c.counts.ensure(sizeof(uint32_t) * radix_scratch_counts(n));
+    c.scan_tmp.ensure(scan_tmp_bytes(std::max<int64_t>(radix_scratch_counts(n), n)));
+    c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
+    c.minord.ensure(sizeof(uint32_t) * kMaxD);
+    c.codes_id.ensure(sizeof(uint16_t) * n * c.dp);
+    c.codes_sorted.ensure(sizeof(uint16_t) * npad * c.dp);
+    c.ord_sorted.ensure(sizeof(uint32_t) * npad * d);
+    c.chunks_all.ensure(sizeof(uint32_t) * (npad / 32) * kRecAll * cw);
+    if (R != c.rbuf.as<uint32_t>())
+        SKY_CUDA(cudaMemcpyAsync(c.rbuf.p, R, sizeof(uint32_t) * d, cudaMemcpyDeviceToDevice, st));
+    if (minord != c.minord.as<uint32_t>())
+        SKY_CUDA(cudaMemcpyAsync(c.minord.p, minord, sizeof(uint32_t) * d, cudaMemcpyDeviceToDevice, st));
+    k2_transpose_kernel<<<blocks_for(n, 256), 256, 0, st>>>(codes_dm, n, d, c.dp, c.codes_id.as<uint16_t>());
+    c.L.count++;
+    SKY_LAUNCH_CHECK();
     SKY_CUDA(cudaMemcpyAsync(c.R, c.rbuf.p, sizeof(uint32_t) * d, cudaMemcpyDeviceToHost, st));
     // static-tree leaf order: Morton key of the codes (top bits first), then chunks of 32
     // (at most 32 key bits: the top bits decide the chunks of 32 and their sub-chunks -- 2^15 chunks at n = 1M --
@@ -423,6 +451,14 @@ void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) 
         c.cshift |= (uint64_t)sh << (4 * i);
     }
     c.prepared = true;
+}
+
+void prep_run(Ctx &c, const float *d_points, int64_t n, int d, cudaStream_t st) {
+    c.codes_dm.ensure(sizeof(uint16_t) * n * d);
+    c.rbuf.ensure(sizeof(uint32_t) * kMaxD);
+    c.minord.ensure(sizeof(uint32_t) * kMaxD);
+    prep_dims(c, d_points, n, d, 0, d, c.codes_dm.as<uint16_t>(), c.rbuf.as<uint32_t>(), c.minord.as<uint32_t>(), st);
+    prep_finish(c, c.codes_dm.as<uint16_t>(), c.rbuf.as<uint32_t>(), c.minord.as<uint32_t>(), st);
 }
 
 void ext_build(Ctx &c, const uint8_t *d_ext_sorted, cudaStream_t st) {

@@ -3,7 +3,10 @@
 Sharding (the paper's device-level data parallelism of MDMC, L308-310, L420 "every
 task is independent, there is no need for synchronisation"):
 
-  1. prepare (K0 + key-sum sort + K2 codes)      replicated on every rank (deterministic, ~2 ms at H)
+  1. prepare                                     K0 on every rank; K2 (per-dimension sort -> dense-rank codes) on
+                                                  the rank's slice of the dimensions (dim_slice), all_gather of the
+                                                  codes (world x ceil(d/world) x n uint16: 24 MB at H) and of the
+                                                  per-dimension counts; the static-tree order replicated
   2. K1 prefilter                                 blocks of 512 static-tree positions, block b on rank b % world
   3. exchange S+ flags                            all_reduce(MAX) of a uint8 flag vector (NCCL over NVLink)
   4. install S+ (replicated)
@@ -39,6 +42,12 @@ GROUP = 32
 def prefilter_assignment(rank: int, world: int):
     """(block_offset, block_step) of the K1 blocks a rank processes."""
     return rank, world
+
+
+def dim_slice(d: int, world: int, rank: int):
+    """[dim_begin, dim_end) of the dimensions whose codes (K2) a rank computes in the sharded prepare."""
+    per = -(-d // world)
+    return min(d, rank * per), min(d, (rank + 1) * per)
 
 
 def task_range(m: int, world: int, rank: int):
@@ -94,6 +103,30 @@ def exchange_totals(totals: torch.Tensor, group=None) -> torch.Tensor:
     else:
         dist.all_gather_into_tensor(out, totals, group=group)
     return out
+
+
+def exchange_codes(mine: torch.Tensor, R: torch.Tensor, minord: torch.Tensor, d: int, group=None):
+    """All-gather the ranks' dimension slices of the codes (each rank [ceil(d/world), n] uint16 as int16, the
+    rows past its slice unused) into [d, n], and combine the per-dimension distinct counts and minimum keys
+    (uint32 [d] as int64, each entry written by exactly one rank, zero elsewhere: a SUM)."""
+    world = _world(group)
+    per, n = mine.shape
+    mb = mine.contiguous().view(torch.uint8)  # 16-bit codes travel as bytes (neither gloo nor NCCL reduce int16)
+    if _staged(mine, group):
+        h = torch.empty((world * per, 2 * n), dtype=torch.uint8)
+        dist.all_gather_into_tensor(h, mb.cpu(), group=group)
+        allc = h.to(mine.device)
+        rm = torch.stack([R, minord]).cpu()
+        dist.all_reduce(rm, op=dist.ReduceOp.SUM, group=group)
+        rm = rm.to(mine.device)
+    else:
+        allc = torch.empty((world * per, 2 * n), dtype=torch.uint8, device=mine.device)
+        dist.all_gather_into_tensor(allc, mb, group=group)
+        rm = torch.stack([R, minord])
+        dist.all_reduce(rm, op=dist.ReduceOp.SUM, group=group)
+    allc = allc.view(mine.dtype)
+    rows = [allc[r * per: r * per + (dim_slice(d, world, r)[1] - dim_slice(d, world, r)[0])] for r in range(world)]
+    return torch.cat(rows).contiguous(), rm[0].to(torch.int32).contiguous(), rm[1].to(torch.int32).contiguous()
 
 
 def gather_rows(rows32: torch.Tensor, m: int, d: int, group=None):
@@ -168,7 +201,20 @@ class DeviceSkycube:
         nsub = 1 << d
 
         rec("t0")
-        self.ctx.prepare(pts.data_ptr(), n, d, sp)
+        if world == 1:
+            self.ctx.prepare(pts.data_ptr(), n, d, sp)
+        else:
+            # K2 sharded by dimension, the codes all-gathered; the uint32 counts / keys travel as int64 (SUM)
+            b, e = dim_slice(d, world, rank)
+            per = -(-d // world)
+            mine = torch.zeros((per, n), dtype=torch.int16, device=self.device)
+            R32 = torch.zeros(d, dtype=torch.int32, device=self.device)
+            mo32 = torch.zeros(d, dtype=torch.int32, device=self.device)
+            self.ctx.prepare_dims(pts.data_ptr(), n, d, b, e, mine.data_ptr(), R32.data_ptr(), mo32.data_ptr(), sp)
+            R64 = R32.to(torch.int64) & 0xffffffff
+            mo64 = mo32.to(torch.int64) & 0xffffffff
+            codes, Rall, moall = exchange_codes(mine, R64, mo64, d, self.group)
+            self.ctx.prepare_finish(codes.data_ptr(), Rall.data_ptr(), moall.data_ptr(), sp)
         rec("t1")
         ext8 = torch.zeros(n, dtype=torch.uint8, device=self.device)
         off, step = prefilter_assignment(rank, world)

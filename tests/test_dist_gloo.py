@@ -158,3 +158,51 @@ def test_sharding_arithmetic():
         for world in [1, 2, 3, 8]:
             sl = [pl.id_slice(n, world, r) for r in range(world)]
             assert sl[0][0] == 0 and sl[-1][1] == n and all(sl[i][1] == sl[i + 1][0] for i in range(world - 1))
+
+
+def _codes_worker(rank, world, port, codes, R, mino, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        d, n = codes.shape
+        b, e = pl.dim_slice(d, world, rank)
+        per = -(-d // world)
+        # K2 stand-in: this rank's slice of the dimension-major codes, counts and minimum keys (zero elsewhere)
+        mine = torch.zeros((per, n), dtype=torch.int16)
+        mine[: e - b] = torch.from_numpy(codes[b:e].astype(np.int16))
+        Rl = torch.zeros(d, dtype=torch.int64)
+        ml = torch.zeros(d, dtype=torch.int64)
+        Rl[b:e] = torch.from_numpy(R[b:e].astype(np.int64))
+        ml[b:e] = torch.from_numpy(mino[b:e].astype(np.int64))
+        allc, Ra, ma = pl.exchange_codes(mine, Rl, ml, d)
+        q.put((rank, allc.numpy().view(np.uint16).copy(), Ra.numpy().view(np.uint32).copy(),
+               ma.numpy().view(np.uint32).copy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,d", [(2, 12), (3, 12), (3, 2), (2, 16), (8, 3)])
+def test_codes_exchange_reassembles_all_dimensions(world, d):
+    """The sharded prepare (pipeline.exchange_codes): every rank computes the codes of its slice of the
+    dimensions; after the all-gather every rank holds the codes of every dimension in dimension order, and the
+    per-dimension counts / minimum keys (uint32, including values above 2^31) of every dimension."""
+    rng = np.random.default_rng(5 + d)
+    n = 1500
+    codes = rng.integers(0, 32768, size=(d, n)).astype(np.uint16)
+    R = rng.integers(1, 2 ** 32, size=d, dtype=np.uint64).astype(np.uint32)
+    mino = rng.integers(0, 2 ** 32, size=d, dtype=np.uint64).astype(np.uint32)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_codes_worker, args=(r, world, port, codes, R, mino, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    sl = [pl.dim_slice(d, world, r) for r in range(world)]
+    assert sl[0][0] == 0 and sl[-1][1] == d and all(sl[i][1] == sl[i + 1][0] for i in range(world - 1))
+    for rank, allc, Ra, ma in res:
+        assert np.array_equal(allc, codes), rank
+        assert np.array_equal(Ra, R) and np.array_equal(ma, mino), rank
