@@ -175,3 +175,42 @@ def test_capi_num_gpus_vs_oracle(tuning, k, name, ref):
         assert r.stats["kernel_launches"] > 0 and r.stats["num_gpus"] == k
     with sky.skycube_build_raw(x, num_gpus=k, max_level=3) as r:
         assert np.array_equal(r.membership(), sky.skycube_build(x, max_level=3)["rows"])
+
+
+def _nccl_worker(port, q):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sigmod_boghcsa17_b200 import pipeline as pl
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        d, n = 12, 1000
+        g = torch.Generator().manual_seed(3)
+        codes = torch.randint(0, 32768, (d, n), generator=g, dtype=torch.int32).to(torch.int16).cuda()
+        R = torch.randint(1, 2 ** 32 - 1, (d,), generator=g, dtype=torch.int64).cuda()
+        mo = torch.randint(0, 2 ** 32 - 1, (d,), generator=g, dtype=torch.int64).cuda()
+        allc, Ra, ma = pl.exchange_codes(codes, R, mo, d)
+        ext8 = torch.randint(0, 2, (n,), generator=g, dtype=torch.uint8).cuda()
+        dist.all_reduce(ext8, op=dist.ReduceOp.MAX)  # the exchange_ext collective on a CUDA uint8 tensor
+        ok = (torch.equal(allc, codes) and torch.equal(Ra.to(torch.int64) & 0xffffffff, R)
+              and torch.equal(ma.to(torch.int64) & 0xffffffff, mo))
+        q.put(bool(ok))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_collectives_single_rank():
+    """The pipeline's collectives on NCCL itself (one rank: this box has one GPU, and NCCL refuses two ranks on one
+    device): the dimension-sharded prepare's codes all-gather (uint16 codes as bytes) and counts all-reduce
+    (int64), and the S+ flag all-reduce(MAX) on uint8 -- the dtypes and call forms the N-GPU run uses."""
+    import torch
+    import torch.multiprocessing as mp
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_worker, args=(_free_port(), q))
+    p.start()
+    ok = q.get(timeout=300)
+    p.join(timeout=60)
+    assert p.exitcode == 0 and ok
