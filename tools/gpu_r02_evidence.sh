@@ -37,7 +37,7 @@ fi
 # per-rank K1 / K3 work of an N-GPU run, measured on this one GPU (tools/k3_shard_time.py)
 for c in ${SHARD_CONFIGS:-H C4}; do for w in 1 2 4 8; do timeout 900 python tools/k3_shard_time.py $c $w 3; done; done \
   > gpurun_out/ev_shards.jsonl 2> gpurun_out/ev_shards.err
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k1_ -c 1 -f -o gpurun_out/ev_prof_k1_H \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k1_prefilter -c 1 -f -o gpurun_out/ev_prof_k1_H \
   python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu --config H > gpurun_out/ev_ncu_k1_H.log 2>&1
 summ ev_prof_k1_H
 cat gpurun_out/ev_tests.log gpurun_out/ev_smoke.log
