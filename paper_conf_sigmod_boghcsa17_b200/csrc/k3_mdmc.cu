@@ -622,8 +622,13 @@ __device__ __forceinline__ void load_row2_s(uint32_t a, uint32_t *w) {
 // warp holds until it has finished the tile.  Needs 32 tasks' state in shared memory (d <= 15).
 // design O's ring: 3 stages with 24 warps (a warp holds its stage until its sub/pair passes are done; C5 K3
 // 20.6 ms with 2 stages, 20.2 with 3)
+// (3 ring stages at d >= 15 too: the one partial group's 16 warps wait less at the tile boundary with a stage more
+// of slack than they lose with one task fewer per CTA -- C4 K3 595.7 -> 576.6 ms; design A keeps 2 there)
+#ifndef SKY_K3_O_STAGES_HIGHD
+#define SKY_K3_O_STAGES_HIGHD 3
+#endif
 template <int D, int MODE, int NW>
-using GeoO = GeoK3<D, MODE, NW, (NW > kWarps && D < 15 ? 3 : 0)>;
+using GeoO = GeoK3<D, MODE, NW, (D >= 15 ? SKY_K3_O_STAGES_HIGHD : NW > kWarps ? 3 : 0)>;
 
 template <int D, int MODE, int NW>
 __global__ void __launch_bounds__((NW + 1) * 32, 1) k3_owner_kernel(
